@@ -1,0 +1,105 @@
+"""a1 — logical tree construction (oracle; test infrastructure only).
+
+Paper basis
+  * Tree AllReduce: "reduction as data moves up the tree and broadcast as data
+    moves down the tree"; the 4-node worked example has root N4 <- N2 <- {N1, N3}
+    (§III-A, Fig 5(a)).
+  * Double binary tree [45]: "a double binary tree ... is commonly used with two
+    trees" (§III-B) and "the first tree is flipped to invert the nodes and
+    leaves to create the second tree" (fn4).
+
+Reading R1: tree 0 is the binary tree rooted at rank 0 with a
+single child; every other rank r with lowest set bit b has parent
+``(r ^ b) | (b << 1)`` or, if that is >= P, ``r ^ b``.  At P=4 this is exactly the
+paper's example 0 <- 2 <- {1, 3} (ranks = N_i - 1 with N4 the root relabelled 0).
+Tree 1 relabels tree 0 by phi(v) = P-1-v for even P (the "flip": tree-0 leaves
+become tree-1 interior nodes) and phi(v) = (v+1) mod P for odd P.
+Children are listed in ascending rank; that order is the combine order (R2).
+"""
+
+from dataclasses import dataclass
+from typing import List, Tuple
+
+
+@dataclass(frozen=True)
+class Tree:
+    P: int
+    root: int
+    parent: Tuple[int, ...]                 # parent[v], -1 at the root
+    children: Tuple[Tuple[int, ...], ...]   # children[v], ascending rank
+
+    def depth(self) -> int:
+        """Depth in edges = max over v of the path length to the root."""
+        best = 0
+        for v in range(self.P):
+            d, u = 0, v
+            while self.parent[u] != -1:
+                u = self.parent[u]
+                d += 1
+            best = max(best, d)
+        return best
+
+    def leaves(self) -> List[int]:
+        return [v for v in range(self.P) if not self.children[v]]
+
+    def interior(self) -> List[int]:
+        """Ranks with at least one child (the root included)."""
+        return [v for v in range(self.P) if self.children[v]]
+
+
+def _lowest_set_bit(r: int) -> int:
+    return r & -r
+
+
+def btree_parent(r: int, P: int) -> int:
+    """Parent of rank r in tree 0 (R1).  Rank 0 is the root."""
+    if r == 0:
+        return -1
+    b = _lowest_set_bit(r)
+    up = (r ^ b) | (b << 1)
+    return up if up < P else (r ^ b)
+
+
+def _from_parent(P: int, parent: List[int]) -> Tree:
+    children: List[List[int]] = [[] for _ in range(P)]
+    root = -1
+    for v in range(P):
+        if parent[v] == -1:
+            root = v
+        else:
+            children[parent[v]].append(v)
+    return Tree(P=P, root=root, parent=tuple(parent),
+                children=tuple(tuple(sorted(c)) for c in children))
+
+
+def tree0(P: int) -> Tree:
+    """The single (first) binary tree, rooted at rank 0."""
+    if P < 1:
+        raise ValueError("P must be >= 1")
+    return _from_parent(P, [btree_parent(r, P) for r in range(P)])
+
+
+def relabel(P: int, v: int) -> int:
+    """phi: tree-0 position v -> rank in tree 1 (R1; fn4 P:L153)."""
+    if P % 2 == 0:
+        return P - 1 - v
+    return (v + 1) % P
+
+
+def tree1(P: int) -> Tree:
+    """The second tree of the double tree: tree 0 with every rank v renamed phi(v)."""
+    t0 = tree0(P)
+    parent = [-1] * P
+    for v in range(P):
+        pv = t0.parent[v]
+        parent[relabel(P, v)] = -1 if pv == -1 else relabel(P, pv)
+    return _from_parent(P, parent)
+
+
+def trees(P: int, kind: str) -> List[Tree]:
+    """kind = 'single' -> [tree0]; 'double' -> [tree0, tree1]."""
+    if kind == "single":
+        return [tree0(P)]
+    if kind == "double":
+        return [tree0(P), tree1(P)]
+    raise ValueError(kind)
