@@ -1,0 +1,398 @@
+#!/usr/bin/env python3
+"""C-Cube bench: tree AllReduce bus bandwidth on B200 (BASELINE.json metric).
+
+N=1 (default): the workload of BASELINE.json configs[1] — the ResNet-50 gradient
+set (25,557,032 fp32, 102,228,128 B per rank) — reduced across P=8 logical ranks
+hosted on ONE B200 ("loopback": the same kernel body that runs one process per
+GPU; every rank's buffer lives in local HBM).  One step = one
+ccube_allreduce_tree_local call = one kernel launch = the whole hot path (a3-a8:
+chunking, reduce-up, C1 turnaround, broadcast-down, enqueue semaphores).
+
+N>1 (torchrun, one process per GPU): P = N real ranks, each with its own
+102 MB buffer, peers mapped over NVLink/NVSwitch with CUDA IPC.
+
+busbw = algbw * 2(P-1)/P with algbw = bytes_per_rank / t (nccl-tests
+convention), t = device time (CUDA events on the launching stream; max over
+ranks for N>1).  --impl reference times the CPU oracle (oracle/) instead.
+"""
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "AllReduce busbw GB/s vs size at 2/4/8 B200 (% of 900 GB/s); iter time chained vs unchained"
+NVLINK_NOMINAL_GBS = 900.0
+NVLINK_MEASURED_GBS = 770.0   # B200_PROFILING.md: measured peer copy per direction
+
+
+def parse():
+    p = argparse.ArgumentParser()
+    p.add_argument("--gpus", type=int, default=1)
+    p.add_argument("--steps", type=int, default=200)
+    p.add_argument("--warmup", type=int, default=10)
+    p.add_argument("--impl", choices=["ccube", "reference"], default="ccube")
+    p.add_argument("--workload", choices=["resnet50", "vgg16"], default="resnet50")
+    p.add_argument("--dtype", choices=["float32", "bfloat16", "int32"], default=None)
+    p.add_argument("--tree", choices=["single", "double"], default=None)
+    p.add_argument("--ranks", type=int, default=8, help="logical ranks in loopback (N=1)")
+    p.add_argument("--overlap", type=int, default=1, help="1 = C1, 0 = B")
+    p.add_argument("--chunk-bytes", type=int, default=256 << 10)
+    p.add_argument("--channels", type=int, default=0)
+    p.add_argument("--threads", type=int, default=0)
+    p.add_argument("--e2e-steps", type=int, default=5)
+    p.add_argument("--no-e2e", action="store_true")
+    p.add_argument("--no-cpu-baseline", action="store_true")
+    p.add_argument("--no-clocks", action="store_true")
+    p.add_argument("--cpu-sample-chunks", type=int, default=0,
+                   help="chunks per step for the oracle (0 = auto)")
+    a = p.parse_args()
+    if a.dtype is None:
+        a.dtype = "bfloat16" if a.workload == "vgg16" else "float32"
+    if a.tree is None:
+        a.tree = "double" if a.workload == "vgg16" else "single"
+    return a
+
+
+def measured_peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured"
+    except Exception:  # noqa: BLE001
+        return 6650.0, "fallback (B200_PROFILING.md)"
+
+
+# ------------------------------------------------------------------------ clocks
+class ClockSampler:
+    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, device_index=0, enabled=True):
+        self.proc = None
+        self.path = os.path.join("/tmp", f"ccube_clocks_{os.getpid()}.csv")
+        self.dev = device_index
+        if enabled:
+            try:
+                self.proc = subprocess.Popen(
+                    ["nvidia-smi", "-i", str(device_index), f"--query-gpu={self.FIELDS}",
+                     "--format=csv,noheader,nounits", "-lms", "100"],
+                    stdout=open(self.path, "w"), stderr=subprocess.DEVNULL)
+            except Exception:  # noqa: BLE001
+                self.proc = None
+
+    def stop(self):
+        if self.proc is None:
+            return None
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:  # noqa: BLE001
+            self.proc.kill()
+        rows = []
+        for line in open(self.path):
+            parts = [x.strip() for x in line.split(",")]
+            if len(parts) < 9:
+                continue
+            try:
+                rows.append(parts)
+            except Exception:  # noqa: BLE001
+                pass
+        if not rows:
+            return None
+        sm = [float(r[1]) for r in rows if r[1].replace(".", "").isdigit()]
+        smax = [float(r[2]) for r in rows if r[2].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in rows for i in range(4)
+                          if r[5 + i].lower().startswith("active")})
+        return {"sm_mhz": float(np.median(sm)) if sm else None,
+                "sm_max_mhz": max(smax) if smax else None,
+                "reasons": reasons, "samples": len(rows)}
+
+
+# ---------------------------------------------------------------- oracle timing
+def oracle_time(P, tree, dtype, workload, chunk_bytes, nchunks, overlap):
+    """Time the CPU oracle's message-passing replay on the first ``nchunks`` chunks
+    of the workload (every rank's data for those chunks)."""
+    from oracle import allreduce as oar
+    from oracle import arith
+    from paper_conf_hpca_sanghoonsk23_b200 import inputs, workloads
+    ends = workloads.layer_ends(workload)
+    E = chunk_bytes // arith.ELEM_SIZE[dtype]
+    count = min(ends[-1], nchunks * E)
+    xs = [inputs.gradients(r, ends[-1], dtype, layer_ends=ends, lo=0, hi=count) for r in range(P)]
+    t0 = time.perf_counter()
+    oar.replay(xs, tree, chunk_bytes, dtype, overlap=bool(overlap))
+    dt = time.perf_counter() - t0
+    return dt, count * arith.ELEM_SIZE[dtype]
+
+
+def busbw(bytes_per_rank, seconds, P):
+    alg = bytes_per_rank / seconds / 1e9
+    return alg * 2 * (P - 1) / P, alg
+
+
+def run_reference(a):
+    """--impl reference: the CPU oracle as it stands, on the host cores (rank 0 only)."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    P = a.ranks if a.gpus == 1 else a.gpus
+    nchunks = a.cpu_sample_chunks or 16   # 16 chunks x 256 KiB = 4 MiB per rank (configs[0] size)
+    for _ in range(a.warmup):
+        oracle_time(P, a.tree, a.dtype, a.workload, a.chunk_bytes, nchunks, a.overlap)
+    total, nbytes = 0.0, 0
+    for _ in range(a.steps):
+        dt, nbytes = oracle_time(P, a.tree, a.dtype, a.workload, a.chunk_bytes, nchunks, a.overlap)
+        total += dt
+    bw, alg = busbw(nbytes, total / a.steps, P)
+    sample = (f"oracle.allreduce.replay on the first {nchunks} chunks ({nbytes} B per rank) of the "
+              f"{a.workload} gradient set, P={P}, {a.tree} tree, one step = one replay")
+    line = {
+        "impl": "reference", "metric": METRIC, "value": bw, "unit": "GB/s", "n_gpus": a.gpus,
+        "steps": a.steps, "warmup": a.warmup, "ms_per_step": total / a.steps * 1e3,
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": _dt(a.dtype),
+        "data": "synthetic", "config": _config(a, P, nbytes),
+        "cpu_baseline": {"value": bw, "unit": "GB/s", "cores": 1, "kind": "oracle",
+                         "sample": sample},
+        "e2e": {"value": bw, "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+        "algbw": alg,
+    }
+    print(json.dumps(line), flush=True)
+
+
+def _dt(d):
+    return {"float32": "f32", "bfloat16": "bf16", "int32": "i32"}[d]
+
+
+def _config(a, P, bytes_per_rank):
+    return {"workload": f"{a.workload} gradient set, {a.tree} tree, {'C1' if a.overlap else 'B'}"
+                        f", P={P}" + (" logical ranks on 1 GPU (loopback)" if a.gpus == 1 else ""),
+            "P": P, "tree": a.tree, "mode": "C1" if a.overlap else "B",
+            "chunk_bytes": a.chunk_bytes, "bytes_per_rank": bytes_per_rank,
+            "seed": 20230225}
+
+
+# -------------------------------------------------------------------- GPU arm
+def run_ccube(a):
+    import torch
+    import torch.distributed as dist
+    from paper_conf_hpca_sanghoonsk23_b200 import ccube, inputs, workloads
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    multi = world > 1
+    torch.cuda.set_device(local_rank if multi else 0)
+    dev = torch.device("cuda", torch.cuda.current_device())
+    if multi:
+        dist.init_process_group("nccl", device_id=dev)
+    P = world if multi else a.ranks
+    nloc = 1 if multi else P
+
+    ends = workloads.layer_ends(a.workload)
+    count = ends[-1]
+    tdt = {"float32": torch.float32, "bfloat16": torch.bfloat16, "int32": torch.int32}[a.dtype]
+    es = torch.tensor([], dtype=tdt).element_size()
+    nbytes = count * es
+
+    # inputs: seeded synthetic gradients, generated on the host once, resident in HBM
+    my_ranks = [rank] if multi else list(range(P))
+    host = []
+    for r in my_ranks:
+        h = torch.empty(count, dtype=tdt).pin_memory()
+        blk = 1 << 24
+        for lo in range(0, count, blk):
+            hi = min(count, lo + blk)
+            x = inputs.gradients(r, count, a.dtype, layer_ends=ends, lo=lo, hi=hi)
+            t = torch.from_numpy(x.view(np.int16)).view(torch.bfloat16) if a.dtype == "bfloat16" \
+                else torch.from_numpy(x)
+            h[lo:hi].copy_(t)
+        host.append(h)
+    pristine = [h.to(dev) for h in host]
+    bufs = [p.clone() for p in pristine]
+
+    if multi:
+        ccube.init_distributed(dist.group.WORLD, tree=a.tree, chunk_bytes=a.chunk_bytes)
+    else:
+        ccube.init_loopback(P, a.tree, a.chunk_bytes)
+    if a.channels:
+        ccube.set_channels(a.channels)
+    if a.threads:
+        ccube.set_threads(a.threads)
+    ccube.set_overlap(bool(a.overlap))
+    info = ccube.get_info()
+    stream = torch.cuda.Stream()
+
+    def step():
+        if multi:
+            ccube.allreduce_tree(bufs[0], stream=stream)
+        else:
+            ccube.allreduce_tree_local(bufs, stream=stream)
+
+    def restore():
+        with torch.cuda.stream(stream):
+            for b, p in zip(bufs, pristine):
+                b.copy_(p)   # > L2 (126 MB): also flushes L2 between timed iterations
+
+    # warm-up
+    for _ in range(max(3, a.warmup)):
+        restore()
+        step()
+    torch.cuda.synchronize()
+    clocks = ClockSampler(local_rank if multi else 0, enabled=(rank == 0 and not a.no_clocks))
+    time.sleep(0.3)
+    # timed region: K steps, each bracketed by events on the launching stream
+    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+           for _ in range(a.steps)]
+    if multi:
+        dist.barrier()
+    torch.cuda.synchronize()
+    for i in range(a.steps):
+        restore()
+        evs[i][0].record(stream)
+        step()
+        evs[i][1].record(stream)
+    torch.cuda.synchronize()
+    if multi:
+        dist.barrier()
+    ms = [s.elapsed_time(e) for s, e in evs]
+    total_ms = float(np.sum(ms))
+    if multi:
+        t = torch.tensor([total_ms], device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        total_ms = t.item()
+    clk = clocks.stop()
+    ms_step = total_ms / a.steps
+    bw, alg = busbw(nbytes, ms_step / 1e3, P)
+
+    # correctness spot-check of the timed configuration (all ranks identical)
+    ok = True
+    if not multi:
+        ok = all(torch.equal(bufs[r], bufs[0]) for r in range(1, P))
+
+    # ---- e2e: host buffers -> device -> allreduce -> host, through the public API
+    e2e = None
+    if not a.no_e2e:
+        outs = [torch.empty_like(h).pin_memory() for h in host]
+        for _ in range(2):
+            with torch.cuda.stream(stream):
+                for b, h in zip(bufs, host):
+                    b.copy_(h, non_blocking=True)
+            step()
+            with torch.cuda.stream(stream):
+                for o, b in zip(outs, bufs):
+                    o.copy_(b, non_blocking=True)
+        torch.cuda.synchronize()
+        if multi:
+            dist.barrier()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for _ in range(a.e2e_steps):
+            with torch.cuda.stream(stream):
+                for b, h in zip(bufs, host):
+                    b.copy_(h, non_blocking=True)
+            step()
+            with torch.cuda.stream(stream):
+                for o, b in zip(outs, bufs):
+                    o.copy_(b, non_blocking=True)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        e2e_ms = e0.elapsed_time(e1) / a.e2e_steps
+        if multi:
+            t = torch.tensor([e2e_ms], device=dev)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            e2e_ms = t.item()
+        ebw, _ = busbw(nbytes, e2e_ms / 1e3, P)
+        e2e = {"value": ebw, "unit": "GB/s", "ms_per_step": e2e_ms,
+               "h2d_bytes_per_step": nbytes * len(my_ranks),
+               "d2h_bytes_per_step": nbytes * len(my_ranks), "steps": a.e2e_steps}
+
+    # ---- roofline of the (single) kernel
+    hbm_peak, peak_src = measured_peaks()
+    if not multi:
+        alg_bytes = 2 * P * nbytes   # each rank's buffer read once + written once
+        achieved = alg_bytes / (ms_step / 1e3) / 1e9
+        roof = {"bound": "hbm", "achieved": achieved, "peak": hbm_peak, "unit": "GB/s",
+                "frac": achieved / hbm_peak, "traffic": _ncu_traffic(),
+                "peak_source": peak_src,
+                "algorithmic_bytes_per_launch": alg_bytes}
+    else:
+        port = max(_port_loads(P, a.tree)) * nbytes
+        achieved = port / (ms_step / 1e3) / 1e9
+        roof = {"bound": "nvlink", "achieved": achieved, "peak": NVLINK_MEASURED_GBS,
+                "unit": "GB/s", "frac": achieved / NVLINK_MEASURED_GBS, "traffic": None,
+                "peak_source": "B200_PROFILING.md measured peer copy per direction",
+                "algorithmic_bytes_per_launch": port}
+
+    cpu = None
+    if rank == 0 and not a.no_cpu_baseline:
+        nch = a.cpu_sample_chunks or 64
+        dt, sb = oracle_time(P, a.tree, a.dtype, a.workload, a.chunk_bytes, nch, a.overlap)
+        cbw, _ = busbw(sb, dt, P)
+        cpu = {"value": cbw, "unit": "GB/s", "cores": 1, "kind": "oracle",
+               "sample": f"oracle.allreduce.replay on the first {nch} chunks ({sb} B per rank) "
+                         f"of the {a.workload} gradient set, P={P}, {a.tree} tree; {dt:.2f} s"}
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": bw, "unit": "GB/s", "n_gpus": world,
+            "steps": a.steps, "warmup": a.warmup, "ms_per_step": ms_step,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+            "dtype": _dt(a.dtype), "data": "synthetic",
+            "config": dict(_config(a, P, nbytes), channels=info["channels"],
+                           threads=info["threads"],
+                           l2="inputs (P x bytes_per_rank) larger than L2 and restored from a "
+                              "pristine copy between timed steps (flushes L2)"),
+            "algbw": alg, "busbw_frac_of_900": bw / NVLINK_NOMINAL_GBS,
+            "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "clocks": clk,
+            "gpu_launches": a.steps, "ranks_identical": ok,
+            "ms_per_step_p10_p50_p90": [float(np.percentile(ms, q)) for q in (10, 50, 90)],
+        }
+        print(json.dumps(line), flush=True)
+    ccube.finalize()
+    if multi:
+        dist.destroy_process_group()
+
+
+def _port_loads(P, kind):
+    """Bytes each rank sends per direction per byte of buffer (library trees)."""
+    from paper_conf_hpca_sanghoonsk23_b200 import ccube
+    ntrees = 2 if kind == "double" else 1
+    loads = [0.0] * P
+    for t in range(ntrees):
+        par = ccube.tree_parents(P, kind, t)
+        for v in range(P):
+            nchild = sum(1 for u in range(P) if par[u] == v)
+            loads[v] += (nchild + (1 if par[v] >= 0 else 0)) / ntrees
+    return loads
+
+
+def _ncu_traffic():
+    """dram bytes per launch from the committed ncu --set full capture, if present."""
+    path = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    try:
+        with open(path) as f:
+            return json.load(f).get("dram_bytes_per_launch")
+    except Exception:  # noqa: BLE001
+        return None
+
+
+def main():
+    a = parse()
+    if a.impl == "reference":
+        run_reference(a)
+    else:
+        run_ccube(a)
+
+
+if __name__ == "__main__":
+    main()

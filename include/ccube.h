@@ -1,0 +1,184 @@
+/*
+ * ccube.h — C ABI of the B200-native C-Cube hot path.
+ *
+ * C-Cube (Jo, Son, Kim, HPCA'23; /root/reference/PAPER.md cited as P:Lnnn) is a
+ * chunk-pipelined tree AllReduce (sum) of data-parallel gradients whose reduce-up
+ * and broadcast-down phases overlap per chunk ("C1"), optionally on
+ * two complementary trees (fn4 P:L153), plus a gradient queue that lets
+ * the next iteration's forward layer l start as soon as the chunks holding its
+ * gradients have landed ("C2").
+ *
+ * Everything on the data path runs in hand-written sm_100a kernels that move data
+ * with 128-bit loads/stores into peer GPUs' memory over NVLink 5 / NVSwitch and
+ * synchronise through single-writer monotone 64-bit counters (acquire/release,
+ * .sys scope).  No NCCL call, no CPU fallback.  The library owns its workspace,
+ * peer mappings, trees and Layer-Chunk Table; the caller owns the gradient buffers.
+ *
+ * Process models (ccube_world_t.nlocal):
+ *   nlocal == 1           one process per GPU (torchrun).  Peer memory is mapped
+ *                         with CUDA IPC through the caller's allgather callback.
+ *   nlocal == world_size  "loopback": one process hosts all P logical ranks on ONE
+ *                         GPU; every rank's buffer is local HBM and one kernel
+ *                         launch runs the same per-rank kernel body for all ranks.
+ *                         Used for single-GPU parity tests and the 1-GPU bench.
+ *
+ * Conventions:
+ *   - Collective calls (init, register, allreduce, finalize) must be made by all
+ *     ranks in the same order with the same count/dtype/tree kind, as with NCCL.
+ *     A mismatch hangs the kernels; the device watchdog (CCUBE_WATCHDOG_MS,
+ *     default 10000) then aborts them and the next call returns CCUBE_ERR_TIMEOUT.
+ *   - Stream-ordered and asynchronous: allreduce/gradq_wait only enqueue work on
+ *     `stream` (a cudaStream_t / CUstream handle; NULL = legacy default stream).
+ *   - In place: the reduced result overwrites `buf` ("stored in the same memory
+ *     address as where they started reduction").
+ *   - Errors: every entry point validates its arguments on the host before any
+ *     launch; CUDA failures map to CCUBE_ERR_CUDA; ccube_last_error() returns a
+ *     thread-local message describing the last failure.
+ */
+#ifndef CCUBE_H
+#define CCUBE_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#if defined(__GNUC__)
+#define CCUBE_API __attribute__((visibility("default")))
+#else
+#define CCUBE_API
+#endif
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+  CCUBE_SUCCESS = 0,
+  CCUBE_ERR_INVALID_ARG = -1,
+  CCUBE_ERR_NOT_INITIALIZED = -2,
+  CCUBE_ERR_ALREADY_INITIALIZED = -3,
+  CCUBE_ERR_CUDA = -4,
+  CCUBE_ERR_UNSUPPORTED = -5,
+  CCUBE_ERR_BOOTSTRAP = -6,
+  CCUBE_ERR_TIMEOUT = -7
+} ccube_result_t;
+
+/* Tree kind.  SINGLE: one binary tree rooted at rank 0.  DOUBLE: two
+ * complementary trees, the second "flipped to invert the nodes and leaves"
+ * (fn4 P:L153); chunk c travels on tree c mod 2 (reading R4). */
+typedef enum { CCUBE_TREE_SINGLE = 0, CCUBE_TREE_DOUBLE = 1 } ccube_tree_kind_t;
+
+/* Element type.  int32 adds wrap mod 2^32; fp32 adds are IEEE RN (no FMA, no FTZ);
+ * bf16 is widened to fp32, added in the fixed order and rounded once (RNE) per
+ * tree node (reading R3).  The combine order at a node is own value, then the
+ * children's partial sums in ascending rank (reading R2). */
+typedef enum { CCUBE_INT32 = 0, CCUBE_FLOAT32 = 1, CCUBE_BFLOAT16 = 2 } ccube_dtype_t;
+
+/* Blocking allgather of `bytes` from every process into recv[p * bytes] (p =
+ * process index = rank / nlocal).  Returns 0 on success.  Supplied by the caller
+ * (the Python layer wraps a torch.distributed process group).  Called only from
+ * inside ccube_init, ccube_register_buffers, ccube_deregister_buffers and
+ * ccube_finalize, on the calling thread. */
+typedef int (*ccube_allgather_fn)(void *ctx, const void *send, void *recv, size_t bytes);
+
+typedef struct {
+  int rank;          /* global rank of the first rank hosted by this process      */
+  int nlocal;        /* ranks hosted by this process: 1, or world_size (loopback)  */
+  int world_size;    /* P, 1..CCUBE_MAX_RANKS                                       */
+  int cuda_device;   /* CUDA device ordinal used by this process                   */
+  ccube_allgather_fn allgather;  /* required when nlocal < world_size               */
+  void *ctx;                     /* passed back to allgather                        */
+} ccube_world_t;
+
+#define CCUBE_MAX_RANKS 8
+#define CCUBE_MAX_CHANNELS 64
+#define CCUBE_DEFAULT_CHUNK_BYTES (256u * 1024u) /* 256 chunks for 64 MB */
+
+/* ccube_init — collective.  Builds the tree(s), allocates the
+ * flag workspace in this GPU's HBM, maps every tree neighbour's workspace (CUDA
+ * IPC over NVLink/NVSwitch when nlocal == 1) and zeroes the monotone counters.
+ *   chunk_bytes: bytes per pipelined chunk ("the amount of data that is
+ *     communicated between neighboring nodes in each step", fn3 P:L88); 0 selects
+ *     CCUBE_DEFAULT_CHUNK_BYTES.  Must be a multiple of 16 * channels.
+ * Errors: INVALID_ARG (bad world/tree/chunk, ranks disagree on the config),
+ * ALREADY_INITIALIZED, UNSUPPORTED (world_size > CCUBE_MAX_RANKS, two processes on
+ * one GPU, no peer access), BOOTSTRAP (allgather callback failed), CUDA. */
+CCUBE_API ccube_result_t ccube_init(const ccube_world_t *world, ccube_tree_kind_t tree_kind,
+                          size_t chunk_bytes);
+
+/* ccube_register_buffers — collective when nlocal < world_size.  Makes the
+ * caller's gradient buffer(s) reachable by tree neighbours: the broadcast writes
+ * fully reduced chunks straight into each child's buffer, which IS the gradient
+ * queue (Fig 9).  Also allocates this rank's receive region
+ * (2 x bytes) into which children push their partial sums.
+ *   bufs: nlocal device pointers (bufs[i] = buffer of rank world.rank + i), each
+ *         16-byte aligned, at least `bytes` long, owned by the caller and kept
+ *         alive until ccube_deregister_buffers / ccube_finalize.
+ * ccube_allreduce_tree[_local] registers an unseen buffer implicitly (collective). */
+CCUBE_API ccube_result_t ccube_register_buffers(void *const *bufs, size_t bytes);
+CCUBE_API ccube_result_t ccube_deregister_buffers(void *const *bufs);
+
+/* ccube_allreduce_tree — collective, one-shot: after it completes
+ * on `stream`, buf[0..count) on every rank holds the same tree-ordered sum of all
+ * ranks' inputs.  Per call the host only validates, looks up the registration,
+ * advances the per-tree epoch and launches ONE kernel.  Requires nlocal == 1.
+ *   buf:   16-byte aligned device pointer on cuda_device (count * elemsize bytes).
+ *   count: elements; 0 is a no-op.  world_size == 1 is a no-op. */
+CCUBE_API ccube_result_t ccube_allreduce_tree(void *buf, size_t count, ccube_dtype_t dtype,
+                                    void *stream);
+
+/* Same for all nlocal ranks hosted by this process (loopback: bufs[r] for r in
+ * 0..P-1, one launch). */
+CCUBE_API ccube_result_t ccube_allreduce_tree_local(void *const *bufs, size_t count,
+                                          ccube_dtype_t dtype, void *stream);
+
+/* ccube_gradq_set_layers — the Layer-Chunk Table source: element offset
+ * at which each layer's gradients end, in forward order (nondecreasing).  Layer l
+ * needs the first ceil(layer_end_elems[l] / E) chunks (readings R9, R10). */
+CCUBE_API ccube_result_t ccube_gradq_set_layers(const size_t *layer_end_elems, int n_layers);
+
+/* ccube_gradq_wait — enqueue on `stream` a device-side wait until every chunk that
+ * holds layer `layer_id`'s gradients (per the most recent allreduce) has landed in
+ * this rank's buffer: the "check" of Fig 11 on the Enqueue Semaphore (P:L204,
+ * P:L266).  No host synchronisation; the next kernel on `stream` (layer l's update
+ * / forward) runs once the wait is satisfied.  The Layer Index Counter is the
+ * caller's call order.  Requires nlocal == 1; the _local form takes the local rank
+ * index. */
+CCUBE_API ccube_result_t ccube_gradq_wait(int layer_id, void *stream);
+CCUBE_API ccube_result_t ccube_gradq_wait_local(int local_rank, int layer_id, void *stream);
+
+/* 1 = C1, the root broadcasts chunk k as soon as it is reduced (default,
+ * P:L163); 0 = B, the root broadcasts only after all chunks are reduced (P:L119,
+ * the paper's baseline "B").  Values are bitwise identical. */
+CCUBE_API ccube_result_t ccube_set_overlap(int on);
+
+/* Channels J per tree (CTA slices of every chunk); all ranks must agree.  0 = the
+ * default (CCUBE_CHANNELS env or 8).  Threads per CTA likewise (64..1024). */
+CCUBE_API ccube_result_t ccube_set_channels(int channels);
+CCUBE_API ccube_result_t ccube_set_threads(int threads);
+
+/* Optional landing trace for gradient-turnaround measurements (Fig 14b):
+ * when set, the thread that publishes chunk k of tree t on local rank r also
+ * stores %globaltimer (ns) into trace[((r * ntrees + t) * kmax + k) * J + j].
+ * NULL disables.  Device pointer of nlocal*ntrees*kmax*J uint64. */
+CCUBE_API ccube_result_t ccube_set_trace(uint64_t *trace, size_t kmax);
+
+CCUBE_API ccube_result_t ccube_finalize(void);
+
+CCUBE_API const char *ccube_last_error(void);
+
+/* Introspection (host-only, no CUDA needed). */
+typedef struct {
+  int initialized, world_size, rank, nlocal, ntrees, channels, threads, overlap;
+  size_t chunk_bytes;
+  uint64_t epoch_base[2];
+} ccube_info_t;
+CCUBE_API ccube_result_t ccube_get_info(ccube_info_t *info);
+
+/* The library's own tree builder (host, pure function): parent[v] of tree `tree`
+ * (0 or 1) of `kind` for P ranks, -1 at the root. */
+CCUBE_API ccube_result_t ccube_tree_parents(int P, ccube_tree_kind_t kind, int tree, int *parent);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* CCUBE_H */

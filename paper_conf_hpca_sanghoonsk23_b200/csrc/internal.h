@@ -1,0 +1,98 @@
+// internal.h — host/device shared layout of the C-Cube runtime (not part of the ABI).
+//
+// Workspace per rank (HBM of the GPU that hosts the rank):
+//   flags  : kFlagBytes of single-writer monotone u64 counters, one per 64 B line
+//            flag(tree, kind, channel) — kind kUpHead0/1: "partial of my k-th chunk
+//            is in your receive plane" written by child slot 0/1 into the parent;
+//            kind kEnq: the Enqueue Semaphore (Fig 9) written by the
+//            parent (or by the root itself) after a fully reduced chunk landed.
+//   recv   : per registered buffer, 2 planes x bytes; child slot s of either tree
+//            writes its partial sum of chunk c at plane s, element offset c*E
+//            (the two trees carry disjoint chunks, so they share the planes).
+// Counters are never reset: a call with base B and K_t tree-local chunks drives
+// every counter of tree t to B + K_t; waits are ">= B + k + 1" (Fig 11 "check").
+#pragma once
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __CUDACC__
+#define CCUBE_HD __host__ __device__
+#else
+#define CCUBE_HD
+#endif
+
+namespace ccube {
+
+constexpr int kMaxRanks = 8;
+constexpr int kMaxChannels = 64;
+constexpr int kMaxTrees = 2;
+constexpr int kMaxChildren = 2;
+constexpr int kFlagStride = 64;  // bytes between two counters
+constexpr int kFlagStrideU64 = kFlagStride / 8;
+
+enum FlagKind { kUpHead0 = 0, kUpHead1 = 1, kEnq = 2, kNumFlagKinds = 3 };
+
+CCUBE_HD inline size_t flag_offset(int tree, int kind, int ch) {
+  return ((static_cast<size_t>(tree) * kNumFlagKinds + kind) * kMaxChannels + ch) * kFlagStride;
+}
+constexpr size_t kFlagBytes =
+    static_cast<size_t>(kMaxTrees) * kNumFlagKinds * kMaxChannels * kFlagStride;
+
+enum Dtype { kInt32 = 0, kFloat32 = 1, kBFloat16 = 2 };
+CCUBE_HD inline int elem_size(int dt) { return dt == kBFloat16 ? 2 : 4; }
+
+// Per (local rank, tree): every pointer the kernel body needs.  "peer" pointers
+// are mapped peer memory (CUDA IPC) in multi-process mode and plain local
+// pointers in loopback mode; the kernel cannot tell the difference.
+struct TreeParams {
+  char *buf;                        // own gradient buffer (= the gradient queue)
+  char *recv[kMaxChildren];         // own receive plane for child slot s
+  char *parent_recv;                // parent's receive plane for my slot (peer); null at root
+  char *child_buf[kMaxChildren];    // children's gradient buffers (peer)
+  uint64_t *head_in[kMaxChildren];  // own counters written by child slot s (channel 0)
+  uint64_t *head_out;               // parent's counter for my slot (peer, channel 0)
+  uint64_t *enq;                    // own Enqueue Semaphore (channel 0)
+  uint64_t *child_enq[kMaxChildren];// children's Enqueue Semaphores (peer, channel 0)
+  int nchild;
+  int is_root;
+  int self_local;                   // local index of this rank (trace)
+  int child_local[kMaxChildren];    // local index of each child, -1 if remote (trace)
+};
+
+enum Role { kRoleUp = 0, kRoleDown = 1 };
+
+struct Task {
+  int16_t local_rank;
+  int16_t tree;
+  int16_t role;
+  int16_t channel;
+};
+
+struct LaunchArgs {
+  const Task *tasks;
+  const TreeParams *params;   // [local_rank * ntrees + tree]
+  uint64_t count;             // elements
+  uint32_t elems_per_chunk;   // E
+  uint32_t slice_elems;       // E / J
+  uint32_t ntrees;
+  uint32_t nchannels;
+  uint32_t K[kMaxTrees];      // tree-local chunk counts
+  uint64_t base[kMaxTrees];   // counter base of this call per tree
+  int overlap;                // 1 = C1, 0 = B
+  int pad0;
+  uint64_t timeout_ns;        // watchdog
+  int *err;                   // mapped host word; nonzero = abort
+  uint64_t *trace;            // optional landing trace
+  uint32_t trace_kmax;
+  uint32_t pad1;
+};
+
+// Kernel launcher (tree_allreduce.cu).  Returns a cudaError_t as int.
+int launch_tree_allreduce(const LaunchArgs &args, int dtype, bool sys_scope, int grid,
+                          int threads, void *stream);
+constexpr int kMaxGateCounters = 128;
+int launch_gate(const uint64_t *const *counters, const uint64_t *targets, int n, int *err,
+                uint64_t timeout_ns, bool sys_scope, void *stream);
+int query_max_blocks_per_sm(int dtype, bool sys_scope, int threads, int *blocks);
+
+}  // namespace ccube

@@ -1,0 +1,844 @@
+// runtime.cc — host side of the C-Cube library: the C ABI of include/ccube.h.
+//
+// Per call the host does only argument validation, a registration lookup, the
+// chunk arithmetic of a3 (K = ceil(bytes / chunk_bytes), chunk c on tree c mod T)
+// and ONE kernel launch; everything on the data path runs on the GPU.
+//
+// Bootstrap (a2): in multi-process mode (nlocal < world_size) the caller's
+// allgather callback carries (i) a config-agreement record, (ii) CUDA IPC handles
+// of every rank's flag workspace, and later (iii) handles of registered gradient
+// buffers and receive regions.  Only tree neighbours' handles are opened.  This
+// replaces the paper's GPUDirect P2P setup with NVLink 5 / NVSwitch peer
+// mappings.  In loopback mode (nlocal == world_size) all "peers" are local
+// allocations and no IPC is used.
+#include <cuda.h>
+#include <cuda_runtime.h>
+
+#include <cstdarg>
+#include <cstdint>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <map>
+#include <memory>
+#include <mutex>
+#include <string>
+#include <utility>
+#include <vector>
+
+#include "ccube.h"
+#include "internal.h"
+#include "trees.h"
+
+namespace ccube {
+namespace {
+
+thread_local std::string g_err;
+
+ccube_result_t fail(ccube_result_t code, const char *fmt, ...) {
+  char msg[1024];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(msg, sizeof msg, fmt, ap);
+  va_end(ap);
+  g_err = msg;
+  if (getenv("CCUBE_DEBUG")) fprintf(stderr, "[ccube] error %d: %s\n", code, msg);
+  return code;
+}
+
+#define CUDA_TRY(expr)                                                                      \
+  do {                                                                                      \
+    cudaError_t e_ = (expr);                                                                \
+    if (e_ != cudaSuccess)                                                                  \
+      return fail(CCUBE_ERR_CUDA, "%s failed: %s (%s:%d)", #expr, cudaGetErrorString(e_),  \
+                  __FILE__, __LINE__);                                                      \
+  } while (0)
+
+#define CC_TRY(expr)                         \
+  do {                                       \
+    ccube_result_t r_ = (expr);              \
+    if (r_ != CCUBE_SUCCESS) return r_;      \
+  } while (0)
+
+// ---- driver entry points (no link-time dependency on libcuda) ----------------
+typedef CUresult (*PFN_batchMemOp)(CUstream, unsigned int, CUstreamBatchMemOpParams *,
+                                   unsigned int);
+typedef CUresult (*PFN_getAddressRange)(CUdeviceptr *, size_t *, CUdeviceptr);
+
+struct Driver {
+  PFN_batchMemOp batchMemOp = nullptr;
+  PFN_getAddressRange getAddressRange = nullptr;
+  bool loaded = false;
+};
+Driver g_drv;
+
+void load_driver() {
+  if (g_drv.loaded) return;
+  g_drv.loaded = true;
+  cudaDriverEntryPointQueryResult q;
+  void *fn = nullptr;
+  if (cudaGetDriverEntryPointByVersion("cuStreamBatchMemOp", &fn, 12000, cudaEnableDefault,
+                                       &q) == cudaSuccess &&
+      q == cudaDriverEntryPointSuccess)
+    g_drv.batchMemOp = reinterpret_cast<PFN_batchMemOp>(fn);
+  fn = nullptr;
+  if (cudaGetDriverEntryPointByVersion("cuMemGetAddressRange", &fn, 12000, cudaEnableDefault,
+                                       &q) == cudaSuccess &&
+      q == cudaDriverEntryPointSuccess)
+    g_drv.getAddressRange = reinterpret_cast<PFN_getAddressRange>(fn);
+}
+
+// ---- IPC bookkeeping ---------------------------------------------------------
+struct IpcEntry {
+  cudaIpcMemHandle_t handle;
+  uint64_t offset;
+  uint64_t bytes;
+  int32_t valid;
+  int32_t pad;
+};
+
+struct OpenedHandle {
+  void *base;
+  int refs;
+};
+std::map<std::string, OpenedHandle> g_opened;  // key = raw handle bytes
+
+ccube_result_t ipc_open(const cudaIpcMemHandle_t &h, void **base) {
+  std::string key(reinterpret_cast<const char *>(&h), sizeof h);
+  auto it = g_opened.find(key);
+  if (it != g_opened.end()) {
+    it->second.refs++;
+    *base = it->second.base;
+    return CCUBE_SUCCESS;
+  }
+  void *p = nullptr;
+  CUDA_TRY(cudaIpcOpenMemHandle(&p, h, cudaIpcMemLazyEnablePeerAccess));
+  g_opened[key] = OpenedHandle{p, 1};
+  *base = p;
+  return CCUBE_SUCCESS;
+}
+
+void ipc_close(void *base) {
+  for (auto it = g_opened.begin(); it != g_opened.end(); ++it) {
+    if (it->second.base == base) {
+      if (--it->second.refs == 0) {
+        cudaIpcCloseMemHandle(base);
+        g_opened.erase(it);
+      }
+      return;
+    }
+  }
+}
+
+struct Registration {
+  std::vector<char *> bufs;       // [nlocal] caller-owned
+  size_t bytes = 0;
+  std::vector<char *> recv;       // [nlocal] library-owned, 2 * bytes each
+  std::vector<char *> world_buf;  // [world] usable pointer (local or peer-mapped), or null
+  std::vector<char *> world_recv; // [world]
+  std::vector<void *> opened;     // IPC bases to close
+  TreeParams *d_params = nullptr; // [nlocal * ntrees]
+};
+
+struct TaskTable {
+  Task *d_tasks = nullptr;
+  int n = 0;
+};
+
+struct Comm {
+  bool init = false;
+  bool poisoned = false;
+  int world = 0, rank0 = 0, nlocal = 0, device = 0, nproc = 1, proc = 0;
+  ccube_allgather_fn allgather = nullptr;
+  void *ctx = nullptr;
+  int ntrees = 1;
+  size_t chunk_bytes = CCUBE_DEFAULT_CHUNK_BYTES;
+  Tree trees[kMaxTrees];
+  int channels = 8, threads = 512, overlap = 1;
+  uint64_t base[kMaxTrees] = {0, 0};
+  bool have_call = false;
+  uint64_t last_base[kMaxTrees] = {0, 0};
+  uint32_t last_K[kMaxTrees] = {0, 0};
+  uint64_t last_E = 0;
+  int last_channels = 0;
+  std::vector<size_t> layer_ends;
+  std::vector<char *> flags_local;  // [nlocal]
+  std::vector<char *> world_flags;  // [world]
+  std::vector<void *> opened_flags;
+  int *err_host = nullptr, *err_dev = nullptr;
+  std::vector<std::unique_ptr<Registration>> regs;
+  std::map<std::pair<int, int>, TaskTable> tasks;  // (channels, overlap)
+  bool sys_scope = false;
+  uint64_t timeout_ns = 10000ull * 1000000ull;
+  int sm_count = 0;
+  std::map<std::pair<int, int>, int> max_blocks;  // (dtype, threads)
+  uint64_t *trace = nullptr;
+  size_t trace_kmax = 0;
+  bool use_memop = true;
+};
+
+Comm g;
+std::mutex g_mu;
+
+int env_int(const char *name, int dflt) {
+  const char *v = getenv(name);
+  return v && *v ? atoi(v) : dflt;
+}
+
+bool is_local(int r) { return r >= g.rank0 && r < g.rank0 + g.nlocal; }
+
+bool is_neighbor_of_local(int r) {
+  for (int i = 0; i < g.nlocal; ++i) {
+    const int v = g.rank0 + i;
+    for (int t = 0; t < g.ntrees; ++t) {
+      const Tree &tr = g.trees[t];
+      if (tr.parent[v] == r) return true;
+      for (int s = 0; s < tr.nchild[v]; ++s)
+        if (tr.child[v][s] == r) return true;
+    }
+  }
+  return false;
+}
+
+ccube_result_t do_allgather(const void *send, void *recv, size_t bytes) {
+  if (g.nproc == 1) {
+    memcpy(recv, send, bytes);
+    return CCUBE_SUCCESS;
+  }
+  if (!g.allgather) return fail(CCUBE_ERR_BOOTSTRAP, "no allgather callback");
+  const int rc = g.allgather(g.ctx, send, recv, bytes);
+  if (rc != 0) return fail(CCUBE_ERR_BOOTSTRAP, "allgather callback returned %d", rc);
+  return CCUBE_SUCCESS;
+}
+
+ccube_result_t check_err_word() {
+  if (g.poisoned) return fail(CCUBE_ERR_TIMEOUT, "communicator aborted by an earlier watchdog timeout");
+  if (g.err_host && *reinterpret_cast<volatile int *>(g.err_host) != 0) {
+    volatile int *e = g.err_host;
+    g.poisoned = true;
+    return fail(CCUBE_ERR_TIMEOUT,
+                "device watchdog fired (block %d waited for counter >= %d, saw %d); the "
+                "communicator must be finalized",
+                e[1], e[2], e[3]);
+  }
+  return CCUBE_SUCCESS;
+}
+
+// Exchange one pointer per local rank through CUDA IPC (multi-process) and
+// produce a usable pointer for every neighbour rank.  In loopback mode the local
+// pointers are used directly.
+ccube_result_t exchange_ptrs(const std::vector<char *> &local, size_t bytes,
+                             std::vector<char *> *world_ptrs, std::vector<void *> *opened) {
+  world_ptrs->assign(g.world, nullptr);
+  for (int i = 0; i < g.nlocal; ++i) (*world_ptrs)[g.rank0 + i] = local[i];
+  if (g.nproc == 1) return CCUBE_SUCCESS;
+  load_driver();
+  std::vector<IpcEntry> mine(g.nlocal);
+  for (int i = 0; i < g.nlocal; ++i) {
+    memset(&mine[i], 0, sizeof(IpcEntry));
+    CUdeviceptr base = 0;
+    size_t sz = 0;
+    if (!g_drv.getAddressRange ||
+        g_drv.getAddressRange(&base, &sz, reinterpret_cast<CUdeviceptr>(local[i])) != CUDA_SUCCESS)
+      return fail(CCUBE_ERR_CUDA, "cuMemGetAddressRange failed for %p", (void *)local[i]);
+    CUDA_TRY(cudaIpcGetMemHandle(&mine[i].handle, reinterpret_cast<void *>(base)));
+    mine[i].offset = reinterpret_cast<CUdeviceptr>(local[i]) - base;
+    mine[i].bytes = bytes;
+    mine[i].valid = 1;
+  }
+  std::vector<IpcEntry> all(static_cast<size_t>(g.nproc) * g.nlocal);
+  CC_TRY(do_allgather(mine.data(), all.data(), sizeof(IpcEntry) * g.nlocal));
+  for (int r = 0; r < g.world; ++r) {
+    if (is_local(r) || !is_neighbor_of_local(r)) continue;
+    const IpcEntry &e = all[r];
+    if (!e.valid || e.bytes != bytes)
+      return fail(CCUBE_ERR_INVALID_ARG, "rank %d registered %llu bytes, expected %llu", r,
+                  (unsigned long long)e.bytes, (unsigned long long)bytes);
+    void *b = nullptr;
+    CC_TRY(ipc_open(e.handle, &b));
+    opened->push_back(b);
+    (*world_ptrs)[r] = static_cast<char *>(b) + e.offset;
+  }
+  return CCUBE_SUCCESS;
+}
+
+ccube_result_t build_params(Registration *R) {
+  std::vector<TreeParams> hp(static_cast<size_t>(g.nlocal) * g.ntrees);
+  for (int i = 0; i < g.nlocal; ++i) {
+    const int r = g.rank0 + i;
+    for (int t = 0; t < g.ntrees; ++t) {
+      const Tree &tr = g.trees[t];
+      TreeParams &p = hp[static_cast<size_t>(i) * g.ntrees + t];
+      memset(&p, 0, sizeof p);
+      p.buf = R->bufs[i];
+      p.recv[0] = R->recv[i];
+      p.recv[1] = R->recv[i] + R->bytes;
+      p.nchild = tr.nchild[r];
+      p.is_root = tr.parent[r] < 0;
+      p.self_local = i;
+      char *fl = g.flags_local[i];
+      for (int s = 0; s < kMaxChildren; ++s) {
+        p.head_in[s] = reinterpret_cast<uint64_t *>(fl + flag_offset(t, kUpHead0 + s, 0));
+        p.child_local[s] = -1;
+      }
+      p.enq = reinterpret_cast<uint64_t *>(fl + flag_offset(t, kEnq, 0));
+      const int par = tr.parent[r];
+      if (par >= 0) {
+        const int slot = child_slot(tr, par, r);
+        if (!R->world_recv[par] || !g.world_flags[par])
+          return fail(CCUBE_ERR_BOOTSTRAP, "parent %d of rank %d not mapped", par, r);
+        p.parent_recv = R->world_recv[par] + static_cast<size_t>(slot) * R->bytes;
+        p.head_out =
+            reinterpret_cast<uint64_t *>(g.world_flags[par] + flag_offset(t, kUpHead0 + slot, 0));
+      }
+      for (int s = 0; s < tr.nchild[r]; ++s) {
+        const int c = tr.child[r][s];
+        if (!R->world_buf[c] || !g.world_flags[c])
+          return fail(CCUBE_ERR_BOOTSTRAP, "child %d of rank %d not mapped", c, r);
+        p.child_buf[s] = R->world_buf[c];
+        p.child_enq[s] = reinterpret_cast<uint64_t *>(g.world_flags[c] + flag_offset(t, kEnq, 0));
+        p.child_local[s] = is_local(c) ? c - g.rank0 : -1;
+      }
+    }
+  }
+  CUDA_TRY(cudaMalloc(&R->d_params, sizeof(TreeParams) * hp.size()));
+  CUDA_TRY(cudaMemcpy(R->d_params, hp.data(), sizeof(TreeParams) * hp.size(),
+                      cudaMemcpyHostToDevice));
+  return CCUBE_SUCCESS;
+}
+
+void free_registration(Registration *R) {
+  for (void *b : R->opened) ipc_close(b);
+  R->opened.clear();
+  for (char *p : R->recv)
+    if (p) cudaFree(p);
+  R->recv.clear();
+  if (R->d_params) cudaFree(R->d_params);
+  R->d_params = nullptr;
+}
+
+ccube_result_t do_register(void *const *bufs, size_t bytes, Registration **out) {
+  if (!bufs) return fail(CCUBE_ERR_INVALID_ARG, "bufs is NULL");
+  if (bytes == 0) return fail(CCUBE_ERR_INVALID_ARG, "bytes == 0");
+  for (int i = 0; i < g.nlocal; ++i) {
+    if (!bufs[i]) return fail(CCUBE_ERR_INVALID_ARG, "bufs[%d] is NULL", i);
+    if (reinterpret_cast<uintptr_t>(bufs[i]) % 16)
+      return fail(CCUBE_ERR_INVALID_ARG, "bufs[%d] = %p is not 16-byte aligned", i, bufs[i]);
+  }
+  std::unique_ptr<Registration> R(new Registration);
+  R->bytes = bytes;
+  for (int i = 0; i < g.nlocal; ++i) R->bufs.push_back(static_cast<char *>(bufs[i]));
+  R->recv.assign(g.nlocal, nullptr);
+  for (int i = 0; i < g.nlocal; ++i) {
+    cudaError_t e = cudaMalloc(&R->recv[i], 2 * bytes);
+    if (e != cudaSuccess) {
+      free_registration(R.get());
+      return fail(CCUBE_ERR_CUDA, "cudaMalloc(recv, %zu) failed: %s", 2 * bytes,
+                  cudaGetErrorString(e));
+    }
+  }
+  ccube_result_t rc = exchange_ptrs(R->bufs, bytes, &R->world_buf, &R->opened);
+  if (rc == CCUBE_SUCCESS) rc = exchange_ptrs(R->recv, 2 * bytes, &R->world_recv, &R->opened);
+  if (rc == CCUBE_SUCCESS) rc = build_params(R.get());
+  if (rc != CCUBE_SUCCESS) {
+    free_registration(R.get());
+    return rc;
+  }
+  *out = R.get();
+  g.regs.push_back(std::move(R));
+  return CCUBE_SUCCESS;
+}
+
+Registration *find_registration(void *const *bufs, size_t bytes) {
+  for (auto &R : g.regs) {
+    if (R->bytes < bytes) continue;
+    bool same = true;
+    for (int i = 0; i < g.nlocal && same; ++i) same = R->bufs[i] == bufs[i];
+    if (same) return R.get();
+  }
+  return nullptr;
+}
+
+ccube_result_t get_tasks(int channels, int overlap, TaskTable **out) {
+  auto key = std::make_pair(channels, overlap);
+  auto it = g.tasks.find(key);
+  if (it != g.tasks.end()) {
+    *out = &it->second;
+    return CCUBE_SUCCESS;
+  }
+  std::vector<Task> ts;
+  for (int i = 0; i < g.nlocal; ++i) {
+    const int r = g.rank0 + i;
+    for (int t = 0; t < g.ntrees; ++t) {
+      const Tree &tr = g.trees[t];
+      const bool root = tr.parent[r] < 0;
+      const bool down = tr.nchild[r] > 0 && (!root || !overlap);
+      for (int j = 0; j < channels; ++j)
+        ts.push_back(Task{(int16_t)i, (int16_t)t, (int16_t)kRoleUp, (int16_t)j});
+      if (down)
+        for (int j = 0; j < channels; ++j)
+          ts.push_back(Task{(int16_t)i, (int16_t)t, (int16_t)kRoleDown, (int16_t)j});
+    }
+  }
+  TaskTable tt;
+  tt.n = static_cast<int>(ts.size());
+  CUDA_TRY(cudaMalloc(&tt.d_tasks, sizeof(Task) * ts.size()));
+  CUDA_TRY(cudaMemcpy(tt.d_tasks, ts.data(), sizeof(Task) * ts.size(), cudaMemcpyHostToDevice));
+  g.tasks[key] = tt;
+  *out = &g.tasks[key];
+  return CCUBE_SUCCESS;
+}
+
+ccube_result_t check_chunk_channels(size_t chunk_bytes, int channels) {
+  if (chunk_bytes == 0 || chunk_bytes % (16ull * channels))
+    return fail(CCUBE_ERR_INVALID_ARG,
+                "chunk_bytes (%zu) must be a positive multiple of 16 * channels (%d)",
+                chunk_bytes, channels);
+  if (chunk_bytes > (1ull << 31))
+    return fail(CCUBE_ERR_INVALID_ARG, "chunk_bytes (%zu) too large", chunk_bytes);
+  return CCUBE_SUCCESS;
+}
+
+ccube_result_t allreduce_impl(void *const *bufs, size_t count, ccube_dtype_t dtype,
+                              void *stream) {
+  if (!g.init) return fail(CCUBE_ERR_NOT_INITIALIZED, "ccube_init has not been called");
+  CC_TRY(check_err_word());
+  if (dtype != CCUBE_INT32 && dtype != CCUBE_FLOAT32 && dtype != CCUBE_BFLOAT16)
+    return fail(CCUBE_ERR_INVALID_ARG, "bad dtype %d", (int)dtype);
+  if (!bufs) return fail(CCUBE_ERR_INVALID_ARG, "bufs is NULL");
+  for (int i = 0; i < g.nlocal; ++i) {
+    if (!bufs[i]) return fail(CCUBE_ERR_INVALID_ARG, "buffer %d is NULL", i);
+    if (reinterpret_cast<uintptr_t>(bufs[i]) % 16)
+      return fail(CCUBE_ERR_INVALID_ARG, "buffer %d (%p) is not 16-byte aligned", i, bufs[i]);
+  }
+  const int es = elem_size(dtype);
+  if (count > (~0ull) / 4) return fail(CCUBE_ERR_INVALID_ARG, "count too large");
+  if (g.world == 1 || count == 0) return CCUBE_SUCCESS;
+  const size_t bytes = count * es;
+  Registration *R = find_registration(bufs, bytes);
+  if (!R) CC_TRY(do_register(bufs, bytes, &R));
+
+  const uint64_t E = g.chunk_bytes / es;
+  const uint64_t K = (count + E - 1) / E;
+  LaunchArgs a;
+  memset(&a, 0, sizeof a);
+  a.count = count;
+  a.elems_per_chunk = static_cast<uint32_t>(E);
+  a.slice_elems = static_cast<uint32_t>(E / g.channels);
+  a.ntrees = g.ntrees;
+  a.nchannels = g.channels;
+  if (g.ntrees == 1) {
+    a.K[0] = static_cast<uint32_t>(K);
+  } else {
+    a.K[0] = static_cast<uint32_t>((K + 1) / 2);
+    a.K[1] = static_cast<uint32_t>(K / 2);
+  }
+  if (K > 0xffffffffull) return fail(CCUBE_ERR_INVALID_ARG, "too many chunks");
+  for (int t = 0; t < g.ntrees; ++t) a.base[t] = g.base[t];
+  a.overlap = g.overlap;
+  a.timeout_ns = g.timeout_ns;
+  a.err = g.err_dev;
+  a.trace = g.trace;
+  a.trace_kmax = static_cast<uint32_t>(g.trace_kmax);
+  a.params = R->d_params;
+
+  TaskTable *tt = nullptr;
+  CC_TRY(get_tasks(g.channels, g.overlap, &tt));
+  a.tasks = tt->d_tasks;
+
+  // all CTAs spin on each other: they must be co-resident
+  auto key = std::make_pair((int)dtype, g.threads);
+  if (!g.max_blocks.count(key)) {
+    int b = 0;
+    const int rc = query_max_blocks_per_sm(dtype, g.sys_scope, g.threads, &b);
+    if (rc != cudaSuccess)
+      return fail(CCUBE_ERR_CUDA, "occupancy query failed: %s",
+                  cudaGetErrorString(static_cast<cudaError_t>(rc)));
+    g.max_blocks[key] = b;
+  }
+  const int cap = g.max_blocks[key] * g.sm_count;
+  if (tt->n > cap)
+    return fail(CCUBE_ERR_UNSUPPORTED,
+                "%d CTAs (channels=%d) cannot be co-resident (capacity %d); lower channels",
+                tt->n, g.channels, cap);
+
+  const int rc = launch_tree_allreduce(a, dtype, g.sys_scope, tt->n, g.threads, stream);
+  if (rc != cudaSuccess)
+    return fail(CCUBE_ERR_CUDA, "kernel launch failed: %s",
+                cudaGetErrorString(static_cast<cudaError_t>(rc)));
+  g.have_call = true;
+  g.last_E = E;
+  g.last_channels = g.channels;
+  for (int t = 0; t < g.ntrees; ++t) {
+    g.last_base[t] = g.base[t];
+    g.last_K[t] = a.K[t];
+    g.base[t] += a.K[t];
+  }
+  return CCUBE_SUCCESS;
+}
+
+ccube_result_t gradq_wait_impl(int local_rank, int layer_id, void *stream) {
+  if (!g.init) return fail(CCUBE_ERR_NOT_INITIALIZED, "ccube_init has not been called");
+  CC_TRY(check_err_word());
+  if (local_rank < 0 || local_rank >= g.nlocal)
+    return fail(CCUBE_ERR_INVALID_ARG, "local_rank %d out of range", local_rank);
+  if (layer_id < 0 || layer_id >= static_cast<int>(g.layer_ends.size()))
+    return fail(CCUBE_ERR_INVALID_ARG, "layer_id %d out of range (%zu layers set)", layer_id,
+                g.layer_ends.size());
+  if (g.world == 1 || !g.have_call) return CCUBE_SUCCESS;
+  // LCT[l] = ceil(end_l / E) chunks (R9, R10); tree t needs its share (R4)
+  const uint64_t total_K = g.ntrees == 1 ? g.last_K[0] : g.last_K[0] + g.last_K[1];
+  uint64_t lct = (g.layer_ends[layer_id] + g.last_E - 1) / g.last_E;
+  if (lct > total_K) lct = total_K;
+  uint64_t need[kMaxTrees] = {lct, 0};
+  if (g.ntrees == 2) {
+    need[0] = (lct + 1) / 2;
+    need[1] = lct / 2;
+  }
+  std::vector<const uint64_t *> ctr;
+  std::vector<uint64_t> tgt;
+  for (int t = 0; t < g.ntrees; ++t) {
+    if (need[t] == 0) continue;
+    for (int j = 0; j < g.last_channels; ++j) {
+      ctr.push_back(reinterpret_cast<const uint64_t *>(g.flags_local[local_rank] +
+                                                       flag_offset(t, kEnq, j)));
+      tgt.push_back(g.last_base[t] + need[t]);
+    }
+  }
+  if (ctr.empty()) return CCUBE_SUCCESS;
+  if (g.use_memop) {
+    load_driver();
+    if (g_drv.batchMemOp) {
+      std::vector<CUstreamBatchMemOpParams> ops(ctr.size());
+      for (size_t i = 0; i < ctr.size(); ++i) {
+        memset(&ops[i], 0, sizeof ops[i]);
+        ops[i].waitValue.operation = CU_STREAM_MEM_OP_WAIT_VALUE_64;
+        ops[i].waitValue.address = reinterpret_cast<CUdeviceptr>(ctr[i]);
+        ops[i].waitValue.value64 = tgt[i];
+        ops[i].waitValue.flags = CU_STREAM_WAIT_VALUE_GEQ;
+      }
+      const CUresult cr = g_drv.batchMemOp(static_cast<CUstream>(stream),
+                                           static_cast<unsigned>(ops.size()), ops.data(), 0);
+      if (cr == CUDA_SUCCESS) return CCUBE_SUCCESS;
+    }
+    g.use_memop = false;  // fall back to the spin-gate kernel from now on
+  }
+  const int rc = launch_gate(ctr.data(), tgt.data(), static_cast<int>(ctr.size()), g.err_dev,
+                             g.timeout_ns, g.sys_scope, stream);
+  if (rc != cudaSuccess)
+    return fail(CCUBE_ERR_CUDA, "gate launch failed: %s",
+                cudaGetErrorString(static_cast<cudaError_t>(rc)));
+  return CCUBE_SUCCESS;
+}
+
+void release_all() {
+  for (auto &R : g.regs) free_registration(R.get());
+  g.regs.clear();
+  for (void *b : g.opened_flags) ipc_close(b);
+  g.opened_flags.clear();
+  for (char *f : g.flags_local)
+    if (f) cudaFree(f);
+  g.flags_local.clear();
+  g.world_flags.clear();
+  for (auto &kv : g.tasks) cudaFree(kv.second.d_tasks);
+  g.tasks.clear();
+  if (g.err_host) cudaFreeHost(g.err_host);
+  g.err_host = g.err_dev = nullptr;
+  g.max_blocks.clear();
+}
+
+struct Hello {
+  uint32_t magic;
+  int32_t world, nlocal, rank, tree_kind, device;
+  uint64_t chunk_bytes;
+  char busid[32];
+};
+
+}  // namespace
+}  // namespace ccube
+
+using namespace ccube;
+
+extern "C" {
+
+ccube_result_t ccube_init(const ccube_world_t *world, ccube_tree_kind_t tree_kind,
+                          size_t chunk_bytes) {
+  std::lock_guard<std::mutex> lk(g_mu);
+  if (g.init) return fail(CCUBE_ERR_ALREADY_INITIALIZED, "already initialized");
+  if (!world) return fail(CCUBE_ERR_INVALID_ARG, "world is NULL");
+  const int P = world->world_size;
+  if (P < 1) return fail(CCUBE_ERR_INVALID_ARG, "world_size %d < 1", P);
+  if (P > CCUBE_MAX_RANKS)
+    return fail(CCUBE_ERR_UNSUPPORTED, "world_size %d > %d (one NVSwitch domain)", P,
+                CCUBE_MAX_RANKS);
+  if (world->nlocal < 1 || P % world->nlocal)
+    return fail(CCUBE_ERR_INVALID_ARG, "nlocal %d must divide world_size %d", world->nlocal, P);
+  if (world->rank < 0 || world->rank >= P || world->rank % world->nlocal)
+    return fail(CCUBE_ERR_INVALID_ARG, "rank %d must be a multiple of nlocal in [0, %d)",
+                world->rank, P);
+  if (tree_kind != CCUBE_TREE_SINGLE && tree_kind != CCUBE_TREE_DOUBLE)
+    return fail(CCUBE_ERR_INVALID_ARG, "bad tree kind %d", (int)tree_kind);
+  if (world->nlocal < P && !world->allgather)
+    return fail(CCUBE_ERR_INVALID_ARG, "allgather callback required when nlocal < world_size");
+  if (chunk_bytes == 0) chunk_bytes = CCUBE_DEFAULT_CHUNK_BYTES;
+  int channels = env_int("CCUBE_CHANNELS", 8);
+  if (channels < 1 || channels > CCUBE_MAX_CHANNELS)
+    return fail(CCUBE_ERR_INVALID_ARG, "CCUBE_CHANNELS %d out of range", channels);
+  CC_TRY(check_chunk_channels(chunk_bytes, channels));
+  int threads = env_int("CCUBE_THREADS", 512);
+  if (threads < 64 || threads > 512 || threads % 32)
+    return fail(CCUBE_ERR_INVALID_ARG, "CCUBE_THREADS %d out of range [64, 512]", threads);
+
+  g = Comm();
+  g.world = P;
+  g.rank0 = world->rank;
+  g.nlocal = world->nlocal;
+  g.device = world->cuda_device;
+  g.nproc = P / world->nlocal;
+  g.proc = world->rank / world->nlocal;
+  g.allgather = world->allgather;
+  g.ctx = world->ctx;
+  g.ntrees = tree_kind == CCUBE_TREE_DOUBLE ? 2 : 1;
+  g.chunk_bytes = chunk_bytes;
+  g.channels = channels;
+  g.threads = threads;
+  g.overlap = 1;
+  g.sys_scope = g.nproc > 1;
+  g.timeout_ns = static_cast<uint64_t>(env_int("CCUBE_WATCHDOG_MS", 10000)) * 1000000ull;
+  g.use_memop = env_int("CCUBE_GATE_KERNEL", 0) == 0;
+  for (int t = 0; t < g.ntrees; ++t) build_tree(P, t, &g.trees[t]);
+
+  // (i) config agreement — host only, so it also runs (and can be tested) without a GPU
+  Hello mine;
+  memset(&mine, 0, sizeof mine);
+  mine.magic = 0xCC0BE001u;
+  mine.world = P;
+  mine.nlocal = g.nlocal;
+  mine.rank = g.rank0;
+  mine.tree_kind = tree_kind;
+  mine.device = g.device;
+  mine.chunk_bytes = chunk_bytes;
+  if (cudaDeviceGetPCIBusId(mine.busid, sizeof mine.busid, g.device) != cudaSuccess)
+    snprintf(mine.busid, sizeof mine.busid, "nodevice-%d", g.rank0);
+  std::vector<Hello> all(g.nproc);
+  ccube_result_t rc = do_allgather(&mine, all.data(), sizeof(Hello));
+  if (rc != CCUBE_SUCCESS) {
+    g = Comm();
+    return rc;
+  }
+  for (int p = 0; p < g.nproc; ++p) {
+    const Hello &h = all[p];
+    if (h.magic != mine.magic || h.world != P || h.nlocal != g.nlocal ||
+        h.rank != p * g.nlocal || h.tree_kind != mine.tree_kind ||
+        h.chunk_bytes != mine.chunk_bytes) {
+      g = Comm();
+      return fail(CCUBE_ERR_INVALID_ARG,
+                  "ranks disagree on the configuration (process %d: world %d nlocal %d rank %d "
+                  "tree %d chunk %llu)",
+                  p, h.world, h.nlocal, h.rank, h.tree_kind, (unsigned long long)h.chunk_bytes);
+    }
+    for (int q = 0; q < p; ++q)
+      if (strncmp(all[q].busid, h.busid, sizeof h.busid) == 0 &&
+          strncmp(h.busid, "nodevice", 8) != 0) {
+        g = Comm();
+        return fail(CCUBE_ERR_UNSUPPORTED,
+                    "processes %d and %d share GPU %s: persistent spinning kernels of two "
+                    "processes cannot run concurrently on one GPU",
+                    q, p, h.busid);
+      }
+  }
+
+  // (ii) CUDA setup
+  cudaError_t ce = cudaSetDevice(g.device);
+  if (ce != cudaSuccess) {
+    g = Comm();
+    return fail(CCUBE_ERR_CUDA, "cudaSetDevice(%d): %s", world->cuda_device,
+                cudaGetErrorString(ce));
+  }
+  auto bail = [&](ccube_result_t r) {
+    release_all();
+    g = Comm();
+    return r;
+  };
+  int major = 0;
+  if (cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, g.device) != cudaSuccess ||
+      cudaDeviceGetAttribute(&g.sm_count, cudaDevAttrMultiProcessorCount, g.device) != cudaSuccess)
+    return bail(fail(CCUBE_ERR_CUDA, "device attribute query failed"));
+  if (major != 10)
+    return bail(fail(CCUBE_ERR_UNSUPPORTED, "compute capability %d.x: built for sm_100a only",
+                     major));
+  ce = cudaHostAlloc(reinterpret_cast<void **>(&g.err_host), 4 * sizeof(int), cudaHostAllocMapped);
+  if (ce != cudaSuccess) return bail(fail(CCUBE_ERR_CUDA, "cudaHostAlloc: %s", cudaGetErrorString(ce)));
+  memset(g.err_host, 0, 4 * sizeof(int));
+  ce = cudaHostGetDevicePointer(reinterpret_cast<void **>(&g.err_dev), g.err_host, 0);
+  if (ce != cudaSuccess) return bail(fail(CCUBE_ERR_CUDA, "cudaHostGetDevicePointer: %s", cudaGetErrorString(ce)));
+  g.flags_local.assign(g.nlocal, nullptr);
+  for (int i = 0; i < g.nlocal; ++i) {
+    ce = cudaMalloc(&g.flags_local[i], kFlagBytes);
+    if (ce == cudaSuccess) ce = cudaMemset(g.flags_local[i], 0, kFlagBytes);
+    if (ce != cudaSuccess) return bail(fail(CCUBE_ERR_CUDA, "flag workspace: %s", cudaGetErrorString(ce)));
+  }
+  ce = cudaDeviceSynchronize();
+  if (ce != cudaSuccess) return bail(fail(CCUBE_ERR_CUDA, "sync: %s", cudaGetErrorString(ce)));
+  g.init = true;  // exchange_ptrs needs the topology fields
+  rc = exchange_ptrs(g.flags_local, kFlagBytes, &g.world_flags, &g.opened_flags);
+  if (rc != CCUBE_SUCCESS) return bail(rc);
+  return CCUBE_SUCCESS;
+}
+
+ccube_result_t ccube_register_buffers(void *const *bufs, size_t bytes) {
+  std::lock_guard<std::mutex> lk(g_mu);
+  if (!g.init) return fail(CCUBE_ERR_NOT_INITIALIZED, "ccube_init has not been called");
+  if (g.world == 1) return CCUBE_SUCCESS;
+  if (bufs && find_registration(bufs, bytes)) return CCUBE_SUCCESS;
+  Registration *R = nullptr;
+  return do_register(bufs, bytes, &R);
+}
+
+ccube_result_t ccube_deregister_buffers(void *const *bufs) {
+  std::lock_guard<std::mutex> lk(g_mu);
+  if (!g.init) return fail(CCUBE_ERR_NOT_INITIALIZED, "ccube_init has not been called");
+  if (!bufs) return fail(CCUBE_ERR_INVALID_ARG, "bufs is NULL");
+  if (g.world == 1) return CCUBE_SUCCESS;
+  for (size_t k = 0; k < g.regs.size(); ++k) {
+    bool same = true;
+    for (int i = 0; i < g.nlocal && same; ++i) same = g.regs[k]->bufs[i] == bufs[i];
+    if (!same) continue;
+    CUDA_TRY(cudaDeviceSynchronize());
+    if (g.nproc > 1) {  // peers must stop using our memory before we unmap theirs
+      std::vector<int> dummy(g.nproc);
+      int one = 1;
+      CC_TRY(do_allgather(&one, dummy.data(), sizeof(int)));
+    }
+    free_registration(g.regs[k].get());
+    g.regs.erase(g.regs.begin() + k);
+    return CCUBE_SUCCESS;
+  }
+  return fail(CCUBE_ERR_INVALID_ARG, "buffer not registered");
+}
+
+ccube_result_t ccube_allreduce_tree(void *buf, size_t count, ccube_dtype_t dtype, void *stream) {
+  std::lock_guard<std::mutex> lk(g_mu);
+  if (g.init && g.nlocal != 1)
+    return fail(CCUBE_ERR_INVALID_ARG,
+                "this process hosts %d ranks: use ccube_allreduce_tree_local", g.nlocal);
+  void *bufs[1] = {buf};
+  return allreduce_impl(bufs, count, dtype, stream);
+}
+
+ccube_result_t ccube_allreduce_tree_local(void *const *bufs, size_t count, ccube_dtype_t dtype,
+                                          void *stream) {
+  std::lock_guard<std::mutex> lk(g_mu);
+  return allreduce_impl(bufs, count, dtype, stream);
+}
+
+ccube_result_t ccube_gradq_set_layers(const size_t *layer_end_elems, int n_layers) {
+  std::lock_guard<std::mutex> lk(g_mu);
+  if (!g.init) return fail(CCUBE_ERR_NOT_INITIALIZED, "ccube_init has not been called");
+  if (n_layers < 0 || (n_layers > 0 && !layer_end_elems))
+    return fail(CCUBE_ERR_INVALID_ARG, "bad layer table");
+  for (int l = 1; l < n_layers; ++l)
+    if (layer_end_elems[l] < layer_end_elems[l - 1])
+      return fail(CCUBE_ERR_INVALID_ARG, "layer_end_elems must be nondecreasing (layer %d)", l);
+  g.layer_ends.assign(layer_end_elems, layer_end_elems + n_layers);
+  return CCUBE_SUCCESS;
+}
+
+ccube_result_t ccube_gradq_wait(int layer_id, void *stream) {
+  std::lock_guard<std::mutex> lk(g_mu);
+  if (g.init && g.nlocal != 1)
+    return fail(CCUBE_ERR_INVALID_ARG, "this process hosts %d ranks: use ccube_gradq_wait_local",
+                g.nlocal);
+  return gradq_wait_impl(0, layer_id, stream);
+}
+
+ccube_result_t ccube_gradq_wait_local(int local_rank, int layer_id, void *stream) {
+  std::lock_guard<std::mutex> lk(g_mu);
+  return gradq_wait_impl(local_rank, layer_id, stream);
+}
+
+ccube_result_t ccube_set_overlap(int on) {
+  std::lock_guard<std::mutex> lk(g_mu);
+  if (!g.init) return fail(CCUBE_ERR_NOT_INITIALIZED, "ccube_init has not been called");
+  if (on != 0 && on != 1) return fail(CCUBE_ERR_INVALID_ARG, "overlap must be 0 or 1");
+  g.overlap = on;
+  return CCUBE_SUCCESS;
+}
+
+ccube_result_t ccube_set_channels(int channels) {
+  std::lock_guard<std::mutex> lk(g_mu);
+  if (!g.init) return fail(CCUBE_ERR_NOT_INITIALIZED, "ccube_init has not been called");
+  if (channels == 0) channels = env_int("CCUBE_CHANNELS", 8);
+  if (channels < 1 || channels > CCUBE_MAX_CHANNELS)
+    return fail(CCUBE_ERR_INVALID_ARG, "channels %d out of range [1, %d]", channels,
+                CCUBE_MAX_CHANNELS);
+  CC_TRY(check_chunk_channels(g.chunk_bytes, channels));
+  g.channels = channels;
+  return CCUBE_SUCCESS;
+}
+
+ccube_result_t ccube_set_threads(int threads) {
+  std::lock_guard<std::mutex> lk(g_mu);
+  if (!g.init) return fail(CCUBE_ERR_NOT_INITIALIZED, "ccube_init has not been called");
+  if (threads < 64 || threads > 512 || threads % 32)
+    return fail(CCUBE_ERR_INVALID_ARG, "threads %d out of range [64, 512] (multiple of 32)",
+                threads);
+  g.threads = threads;
+  return CCUBE_SUCCESS;
+}
+
+ccube_result_t ccube_set_trace(uint64_t *trace, size_t kmax) {
+  std::lock_guard<std::mutex> lk(g_mu);
+  if (!g.init) return fail(CCUBE_ERR_NOT_INITIALIZED, "ccube_init has not been called");
+  if (trace && kmax == 0) return fail(CCUBE_ERR_INVALID_ARG, "kmax == 0");
+  g.trace = trace;
+  g.trace_kmax = trace ? kmax : 0;
+  return CCUBE_SUCCESS;
+}
+
+ccube_result_t ccube_finalize(void) {
+  std::lock_guard<std::mutex> lk(g_mu);
+  if (!g.init) return fail(CCUBE_ERR_NOT_INITIALIZED, "ccube_init has not been called");
+  cudaDeviceSynchronize();
+  ccube_result_t rc = CCUBE_SUCCESS;
+  if (g.nproc > 1) {
+    std::vector<int> dummy(g.nproc);
+    int one = 1;
+    rc = do_allgather(&one, dummy.data(), sizeof(int));
+  }
+  release_all();
+  g = Comm();
+  return rc;
+}
+
+const char *ccube_last_error(void) { return g_err.c_str(); }
+
+ccube_result_t ccube_get_info(ccube_info_t *info) {
+  std::lock_guard<std::mutex> lk(g_mu);
+  if (!info) return fail(CCUBE_ERR_INVALID_ARG, "info is NULL");
+  memset(info, 0, sizeof *info);
+  info->initialized = g.init;
+  info->world_size = g.world;
+  info->rank = g.rank0;
+  info->nlocal = g.nlocal;
+  info->ntrees = g.ntrees;
+  info->channels = g.channels;
+  info->threads = g.threads;
+  info->overlap = g.overlap;
+  info->chunk_bytes = g.chunk_bytes;
+  info->epoch_base[0] = g.base[0];
+  info->epoch_base[1] = g.base[1];
+  return CCUBE_SUCCESS;
+}
+
+ccube_result_t ccube_tree_parents(int P, ccube_tree_kind_t kind, int tree, int *parent) {
+  if (P < 1 || P > kTreeMaxP || !parent) return fail(CCUBE_ERR_INVALID_ARG, "bad P or parent");
+  if (tree < 0 || tree > (kind == CCUBE_TREE_DOUBLE ? 1 : 0))
+    return fail(CCUBE_ERR_INVALID_ARG, "bad tree index %d", tree);
+  Tree t;
+  build_tree(P, tree, &t);
+  for (int v = 0; v < P; ++v) parent[v] = t.parent[v];
+  return CCUBE_SUCCESS;
+}
+
+}  // extern "C"

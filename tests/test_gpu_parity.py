@@ -1,0 +1,278 @@
+"""GPU parity: the CUDA path through the C ABI vs the CPU oracle (loopback mode:
+P logical ranks on one B200, same kernel body as one-process-per-GPU).
+
+Bar (north star / DESIGN.md §5): bit-exact for int32, fp32 and bf16 (same fixed
+order and per-node rounding); every rank identical; B == C1 bitwise; normwise
+error vs an fp64 sum <= 1e-6 (fp32) and <= 1e-2 (bf16)."""
+
+import numpy as np
+import pytest
+import torch
+
+from oracle import allreduce as oar
+from oracle import arith, partition
+from paper_conf_hpca_sanghoonsk23_b200 import ccube, inputs, workloads
+
+from gpu_helpers import device_inputs, oracle_chunk, to_numpy, to_torch
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture
+def comm():
+    """Yields an init function; always finalizes."""
+    state = {"on": False}
+
+    def _init(P, kind="single", chunk_bytes=4096, channels=None, overlap=True, threads=None):
+        ccube.init_loopback(P, kind, chunk_bytes)
+        state["on"] = True
+        if channels is not None:
+            ccube.set_channels(channels)
+        if threads is not None:
+            ccube.set_threads(threads)
+        ccube.set_overlap(overlap)
+
+    yield _init
+    if state["on"]:
+        ccube.finalize()
+
+
+def _run(P, kind, dtype, count, chunk_bytes, seed=5):
+    xs = [inputs.gradients(r, count, dtype, seed=seed) for r in range(P)]
+    ts = [to_torch(x, dtype).cuda() for x in xs]
+    ccube.allreduce_tree_local(ts)
+    torch.cuda.synchronize()
+    return xs, [to_numpy(t, dtype) for t in ts]
+
+
+@pytest.mark.parametrize("P", [2, 3, 4, 5, 8])
+@pytest.mark.parametrize("kind", ["single", "double"])
+@pytest.mark.parametrize("dtype", ["int32", "float32", "bfloat16"])
+@pytest.mark.parametrize("overlap", [True, False])
+def test_parity_small(comm, P, kind, dtype, overlap):
+    """Several chunks (K = 8), 4 channels, ragged tail (not a whole vector)."""
+    chunk = 4096
+    comm(P, kind, chunk, channels=4, overlap=overlap)
+    E = chunk // arith.ELEM_SIZE[dtype]
+    count = 7 * E + 13
+    xs, outs = _run(P, kind, dtype, count, chunk)
+    ref = oar.reference(xs, kind, chunk, dtype)[0]
+    for r in range(P):
+        assert np.array_equal(outs[r], ref), f"rank {r}"
+
+
+@pytest.mark.parametrize("channels", [1, 2, 3, 8, 16])
+def test_parity_channels(comm, channels):
+    chunk = 16 * 1024 * 3   # divisible by 16*channels for all listed channel counts
+    comm(8, "double", chunk, channels=channels)
+    count = 5 * chunk // 4 + 1001
+    xs, outs = _run(8, "double", "float32", count, chunk)
+    ref = oar.reference(xs, "double", chunk, "float32")[0]
+    for r in range(8):
+        assert np.array_equal(outs[r], ref)
+
+
+@pytest.mark.parametrize("threads", [64, 256, 512])
+def test_parity_threads(comm, threads):
+    comm(4, "single", 8192, channels=2, threads=threads)
+    xs, outs = _run(4, "single", "bfloat16", 40000 + 3, 8192)
+    ref = oar.reference(xs, "single", 8192, "bfloat16")[0]
+    for r in range(4):
+        assert np.array_equal(outs[r], ref)
+
+
+def test_repeated_calls_advance_epochs(comm):
+    comm(8, "double", 4096, channels=4)
+    for it in range(4):
+        count = [5000, 20000, 7, 12345][it]
+        xs, outs = _run(8, "double", "float32", count, 4096, seed=100 + it)
+        ref = oar.reference(xs, "double", 4096, "float32")[0]
+        for r in range(8):
+            assert np.array_equal(outs[r], ref), (it, r)
+    info = ccube.get_info()
+    assert info["epoch_base"][0] > 0 and info["epoch_base"][1] > 0
+
+
+@pytest.mark.parametrize("count", [1, 3, 4, 5, 1023, 1024, 1025])
+def test_tiny_and_boundary_counts(comm, count):
+    comm(4, "double", 4096, channels=4)
+    xs, outs = _run(4, "double", "float32", count, 4096)
+    ref = oar.reference(xs, "double", 4096, "float32")[0]
+    for r in range(4):
+        assert np.array_equal(outs[r], ref)
+
+
+def test_count_zero_and_P1_are_noops(comm):
+    comm(4, "single", 4096, channels=4)
+    ts = [torch.arange(100, dtype=torch.float32, device="cuda") + r for r in range(4)]
+    keep = [t.clone() for t in ts]
+    ccube.allreduce_tree_local(ts, count=0)
+    torch.cuda.synchronize()
+    for a, b in zip(ts, keep):
+        assert torch.equal(a, b)
+
+
+def test_P1_loopback_noop():
+    ccube.init_loopback(1, "single", 4096)
+    try:
+        t = torch.arange(100, dtype=torch.float32, device="cuda")
+        ccube.allreduce_tree_local([t])
+        torch.cuda.synchronize()
+        assert torch.equal(t, torch.arange(100, dtype=torch.float32, device="cuda"))
+    finally:
+        ccube.finalize()
+
+
+def test_misaligned_buffer_rejected(comm):
+    comm(2, "single", 4096, channels=4)
+    base = [torch.zeros(1000, dtype=torch.float32, device="cuda") for _ in range(2)]
+    with pytest.raises(ccube.CCubeError) as e:
+        ccube.allreduce_tree_local([b[1:] for b in base])
+    assert e.value.code == ccube.ERR_INVALID_ARG
+    assert "aligned" in ccube.last_error()
+
+
+def test_too_many_channels_rejected(comm):
+    comm(8, "double", 1 << 20, channels=64)
+    ts = [torch.zeros(1 << 20, device="cuda") for _ in range(8)]
+    with pytest.raises(ccube.CCubeError) as e:
+        ccube.allreduce_tree_local(ts)
+    assert e.value.code == ccube.ERR_UNSUPPORTED
+
+
+def test_int32_full_range_wraps(comm):
+    comm(8, "single", 4096, channels=4)
+    count = 9000
+    xs = [inputs.gradients(r, count, "int32", seed=9, full_range=True) for r in range(8)]
+    ts = [to_torch(x, "int32").cuda() for x in xs]
+    ccube.allreduce_tree_local(ts)
+    s = np.zeros(count, dtype=np.int64)
+    for x in xs:
+        s += x.astype(np.int64)
+    want = ((s + 2 ** 31) % 2 ** 32 - 2 ** 31).astype(np.int32)
+    for t in ts:
+        assert np.array_equal(to_numpy(t, "int32"), want)
+
+
+def _full_size(P, kind, dtype, workload, chunk_bytes, overlap=True):
+    ends = workloads.layer_ends(workload)
+    count = ends[-1]
+    ts = device_inputs(P, count, dtype, layer_ends=ends)
+    ccube.set_overlap(overlap)
+    ccube.allreduce_tree_local(ts)
+    torch.cuda.synchronize()
+    return count, ends, ts
+
+
+@pytest.mark.parametrize("kind", ["single", "double"])
+def test_full_size_resnet50_fp32(comm, kind):
+    """configs[1]: ResNet-50 gradient set (25,557,032 fp32, K = 390) at P = 8 with the
+    bench's launch configuration; sampled chunks bit-exact vs the oracle (first,
+    last ragged, random), every rank identical, fp64 normwise error <= 1e-6."""
+    P, chunk = 8, 256 << 10
+    comm(P, kind, chunk)
+    count, ends, ts = _full_size(P, kind, "float32", "resnet50", chunk)
+    K = partition.num_chunks(count, chunk, 4)
+    assert K == 390
+    rng = np.random.default_rng(0)
+    for c in sorted({0, 1, K - 2, K - 1, *rng.integers(0, K, 6).tolist()}):
+        lo, hi, want = oracle_chunk(P, kind, chunk, "float32", count, c, layer_ends=ends)
+        for r in (0, 3, 7):
+            assert np.array_equal(to_numpy(ts[r][lo:hi], "float32"), want), (c, r)
+    for r in range(1, P):
+        assert torch.equal(ts[r], ts[0])
+    # order-independent fp64 reference on the device (a check, not the product path)
+    s = torch.zeros(count, dtype=torch.float64, device="cuda")
+    for x in device_inputs(P, count, "float32", layer_ends=ends):
+        s += x.double()
+    err = (ts[0].double() - s).norm() / s.norm()
+    assert err.item() <= 1e-6
+
+
+def test_full_size_vgg16_bf16_double(comm):
+    """configs[2]: VGG-16 bf16 gradients (138,357,544, K = 1056) on the double tree."""
+    P, chunk = 8, 256 << 10
+    comm(P, "double", chunk)
+    count, ends, ts = _full_size(P, "double", "bfloat16", "vgg16", chunk)
+    K = partition.num_chunks(count, chunk, 2)
+    assert K == 1056
+    for c in (0, 1, 500, 777, K - 2, K - 1):
+        lo, hi, want = oracle_chunk(P, "double", chunk, "bfloat16", count, c, layer_ends=ends)
+        for r in (0, 5):
+            assert np.array_equal(to_numpy(ts[r][lo:hi], "bfloat16"), want), (c, r)
+    for r in range(1, P):
+        assert torch.equal(ts[r], ts[0])
+    s = torch.zeros(count, dtype=torch.float64, device="cuda")
+    for x in device_inputs(P, count, "bfloat16", layer_ends=ends):
+        s += x.double()
+    err = (ts[0].double() - s).norm() / s.norm()
+    assert err.item() <= 1e-2
+
+
+def test_overlap_and_baseline_bitwise_equal_full_size(comm):
+    """P:L272 'C-Cube does not change the ordering of any computation'."""
+    P, chunk = 8, 256 << 10
+    comm(P, "single", chunk)
+    _, _, a = _full_size(P, "single", "float32", "resnet50", chunk, overlap=True)
+    _, _, b = _full_size(P, "single", "float32", "resnet50", chunk, overlap=False)
+    for r in range(P):
+        assert torch.equal(a[r], b[r])
+
+
+@pytest.mark.parametrize("kind", ["single", "double"])
+def test_gradient_queue_gates_each_layer(comm, kind):
+    """a9: on a second stream, gradq_wait(l) then snapshot layer l's gradients; every
+    snapshot must already hold the final reduced values."""
+    P, chunk = 8, 64 << 10
+    comm(P, kind, chunk, channels=4)
+    ends = workloads.layer_ends("resnet50")
+    count = ends[-1]
+    ts = device_inputs(P, count, "float32", layer_ends=ends)
+    ccube.gradq_set_layers(ends)
+    comm_stream = torch.cuda.Stream()
+    comp = torch.cuda.Stream()
+    comm_stream.wait_stream(torch.cuda.current_stream())
+    comp.wait_stream(torch.cuda.current_stream())
+    snaps = {}
+    rank = 5
+    with torch.cuda.stream(comm_stream):
+        ccube.allreduce_tree_local(ts, stream=comm_stream)
+    with torch.cuda.stream(comp):
+        starts = [0] + ends[:-1]
+        for l in range(len(ends)):
+            ccube.gradq_wait_local(rank, l, stream=comp)
+            snaps[l] = ts[rank][starts[l]:ends[l]].clone()
+    torch.cuda.synchronize()
+    final = ts[rank]
+    for l in range(len(ends)):
+        assert torch.equal(snaps[l], final[starts[l]:ends[l]]), f"layer {l} read before landing"
+
+
+def test_landing_trace_in_order_and_c1_turnaround(comm):
+    """Obs #3: chunks land in order per rank/tree/channel; C1 turns the first
+    chunk around long before B (Fig 14(b))."""
+    P, chunk, J = 8, 64 << 10, 4
+    comm(P, "single", chunk, channels=J)
+    count = 64 * chunk // 4
+    K = 64
+    trace = torch.zeros(P * 1 * K * J, dtype=torch.int64, device="cuda")
+    ccube.set_trace(trace, K)
+    ts = device_inputs(P, count, "float32")
+    res = {}
+    for overlap in (False, True):
+        trace.zero_()
+        ccube.set_overlap(overlap)
+        ccube.allreduce_tree_local(ts)
+        torch.cuda.synchronize()
+        tr = trace.view(P, K, J).cpu().numpy().astype(np.int64)
+        assert (tr > 0).all()
+        for r in range(P):
+            for j in range(J):
+                assert np.all(np.diff(tr[r, :, j]) >= 0), (overlap, r, j)
+        land = tr.max(axis=2)                    # a chunk has landed when all slices have
+        t0 = tr.min()
+        res[overlap] = (land[:, 0].max() - t0, land.max() - t0)
+    ccube.set_trace(None, 0)
+    turn_b, total_b = res[False]
+    turn_c, total_c = res[True]
+    assert turn_c * 4 < turn_b, res
