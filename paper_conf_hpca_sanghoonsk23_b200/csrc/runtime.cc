@@ -133,7 +133,8 @@ void ipc_close(void *base) {
 struct Registration {
   std::vector<char *> bufs;       // [nlocal] caller-owned
   size_t bytes = 0;
-  std::vector<char *> recv;       // [nlocal] library-owned, 2 * bytes each
+  size_t plane = 0;               // receive-plane stride: bytes rounded up to 256 B
+  std::vector<char *> recv;       // [nlocal] library-owned, 2 * plane each
   std::vector<char *> world_buf;  // [world] usable pointer (local or peer-mapped), or null
   std::vector<char *> world_recv; // [world]
   std::vector<void *> opened;     // IPC bases to close
@@ -272,7 +273,7 @@ ccube_result_t build_params(Registration *R) {
       memset(&p, 0, sizeof p);
       p.buf = R->bufs[i];
       p.recv[0] = R->recv[i];
-      p.recv[1] = R->recv[i] + R->bytes;
+      p.recv[1] = R->recv[i] + R->plane;
       p.nchild = tr.nchild[r];
       p.is_root = tr.parent[r] < 0;
       p.self_local = i;
@@ -287,7 +288,7 @@ ccube_result_t build_params(Registration *R) {
         const int slot = child_slot(tr, par, r);
         if (!R->world_recv[par] || !g.world_flags[par])
           return fail(CCUBE_ERR_BOOTSTRAP, "parent %d of rank %d not mapped", par, r);
-        p.parent_recv = R->world_recv[par] + static_cast<size_t>(slot) * R->bytes;
+        p.parent_recv = R->world_recv[par] + static_cast<size_t>(slot) * R->plane;
         p.head_out =
             reinterpret_cast<uint64_t *>(g.world_flags[par] + flag_offset(t, kUpHead0 + slot, 0));
       }
@@ -327,18 +328,19 @@ ccube_result_t do_register(void *const *bufs, size_t bytes, Registration **out) 
   }
   std::unique_ptr<Registration> R(new Registration);
   R->bytes = bytes;
+  R->plane = (bytes + 255) & ~static_cast<size_t>(255);
   for (int i = 0; i < g.nlocal; ++i) R->bufs.push_back(static_cast<char *>(bufs[i]));
   R->recv.assign(g.nlocal, nullptr);
   for (int i = 0; i < g.nlocal; ++i) {
-    cudaError_t e = cudaMalloc(&R->recv[i], 2 * bytes);
+    cudaError_t e = cudaMalloc(&R->recv[i], 2 * R->plane);
     if (e != cudaSuccess) {
       free_registration(R.get());
-      return fail(CCUBE_ERR_CUDA, "cudaMalloc(recv, %zu) failed: %s", 2 * bytes,
+      return fail(CCUBE_ERR_CUDA, "cudaMalloc(recv, %zu) failed: %s", 2 * R->plane,
                   cudaGetErrorString(e));
     }
   }
   ccube_result_t rc = exchange_ptrs(R->bufs, bytes, &R->world_buf, &R->opened);
-  if (rc == CCUBE_SUCCESS) rc = exchange_ptrs(R->recv, 2 * bytes, &R->world_recv, &R->opened);
+  if (rc == CCUBE_SUCCESS) rc = exchange_ptrs(R->recv, 2 * R->plane, &R->world_recv, &R->opened);
   if (rc == CCUBE_SUCCESS) rc = build_params(R.get());
   if (rc != CCUBE_SUCCESS) {
     free_registration(R.get());
