@@ -152,9 +152,21 @@ CCUBE_API ccube_result_t ccube_gradq_wait_local(int local_rank, int layer_id, vo
 CCUBE_API ccube_result_t ccube_set_overlap(int on);
 
 /* Channels J per tree (CTA slices of every chunk); all ranks must agree.  0 = the
- * default (CCUBE_CHANNELS env or 8).  Threads per CTA likewise (64..1024). */
+ * default (CCUBE_CHANNELS env or 8).  `threads` = data threads per CTA (32..512,
+ * multiple of 32; CCUBE_THREADS env, default 512); each CTA adds one control warp. */
 CCUBE_API ccube_result_t ccube_set_channels(int channels);
 CCUBE_API ccube_result_t ccube_set_threads(int threads);
+
+/* Edge transport (physical-topology awareness, cf. §IV).  PUSH: a
+ * child stores its partial sum into the parent's receive plane (posted NVLink
+ * writes, the default across GPUs).  PULL: the child keeps its partial in place
+ * in its own buffer and the parent reads it (no receive plane; a leaf moves no
+ * data in the reduce phase).  AUTO = PULL for ranks on the same GPU, PUSH across
+ * GPUs.  Values are bitwise identical for every choice.  All ranks must agree. */
+#define CCUBE_TRANSPORT_AUTO 0
+#define CCUBE_TRANSPORT_PUSH 1
+#define CCUBE_TRANSPORT_PULL 2
+CCUBE_API ccube_result_t ccube_set_transport(int mode);
 
 /* Optional landing trace for gradient-turnaround measurements (Fig 14b):
  * when set, the thread that publishes chunk k of tree t on local rank r also
@@ -168,7 +180,7 @@ CCUBE_API const char *ccube_last_error(void);
 
 /* Introspection (host-only, no CUDA needed). */
 typedef struct {
-  int initialized, world_size, rank, nlocal, ntrees, channels, threads, overlap;
+  int initialized, world_size, rank, nlocal, ntrees, channels, threads, overlap, transport;
   size_t chunk_bytes;
   uint64_t epoch_base[2];
 } ccube_info_t;

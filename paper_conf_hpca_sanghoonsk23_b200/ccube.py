@@ -31,13 +31,14 @@ _NAMES = {0: "SUCCESS", -1: "INVALID_ARG", -2: "NOT_INITIALIZED", -3: "ALREADY_I
           -4: "CUDA", -5: "UNSUPPORTED", -6: "BOOTSTRAP", -7: "TIMEOUT"}
 
 TREE = {"single": 0, "double": 1}
+TRANSPORT = {"auto": 0, "push": 1, "pull": 2}
 DTYPE = {"int32": 0, "float32": 1, "bfloat16": 2}
 
 EXPORTS = [
     "ccube_init", "ccube_register_buffers", "ccube_deregister_buffers", "ccube_allreduce_tree",
     "ccube_allreduce_tree_local", "ccube_gradq_set_layers", "ccube_gradq_wait",
     "ccube_gradq_wait_local", "ccube_set_overlap", "ccube_set_channels", "ccube_set_threads",
-    "ccube_set_trace", "ccube_finalize", "ccube_last_error", "ccube_get_info",
+    "ccube_set_trace", "ccube_set_transport", "ccube_finalize", "ccube_last_error", "ccube_get_info",
     "ccube_tree_parents",
 ]
 
@@ -62,7 +63,7 @@ class Info(ctypes.Structure):
     _fields_ = [("initialized", ctypes.c_int), ("world_size", ctypes.c_int),
                 ("rank", ctypes.c_int), ("nlocal", ctypes.c_int), ("ntrees", ctypes.c_int),
                 ("channels", ctypes.c_int), ("threads", ctypes.c_int), ("overlap", ctypes.c_int),
-                ("chunk_bytes", ctypes.c_size_t), ("epoch_base", ctypes.c_uint64 * 2)]
+                ("transport", ctypes.c_int), ("chunk_bytes", ctypes.c_size_t), ("epoch_base", ctypes.c_uint64 * 2)]
 
 
 _lib = None
@@ -91,6 +92,7 @@ def lib() -> ctypes.CDLL:
             "ccube_set_channels": [i],
             "ccube_set_threads": [i],
             "ccube_set_trace": [vp, sz],
+            "ccube_set_transport": [i],
             "ccube_finalize": [],
             "ccube_get_info": [ctypes.POINTER(Info)],
             "ccube_tree_parents": [i, i, i, ctypes.POINTER(i)],
@@ -263,6 +265,11 @@ def set_channels(channels: int) -> None:
 
 def set_threads(threads: int) -> None:
     _check(lib().ccube_set_threads(threads), "ccube_set_threads")
+
+
+def set_transport(mode: str) -> None:
+    """'auto' (pull inside a GPU, push across GPUs), 'push' or 'pull'."""
+    _check(lib().ccube_set_transport(TRANSPORT[mode]), "ccube_set_transport")
 
 
 def set_trace(trace_tensor, kmax: int) -> None:

@@ -44,10 +44,18 @@ CCUBE_HD inline int elem_size(int dt) { return dt == kBFloat16 ? 2 : 4; }
 // Per (local rank, tree): every pointer the kernel body needs.  "peer" pointers
 // are mapped peer memory (CUDA IPC) in multi-process mode and plain local
 // pointers in loopback mode; the kernel cannot tell the difference.
+//
+// Edge transport (physical-topology reading of §IV): an edge whose
+// two ranks live on different GPUs is PUSH — the child stores its partial sum into
+// the parent's receive plane (posted NVLink writes).  An edge inside one GPU is
+// PULL — the child leaves its partial in place in its own buffer and the parent
+// reads it from there (no receive plane, no extra copy; a pulled leaf moves no
+// data at all in the reduce phase).  Both run the same kernel body; only the
+// pointers below differ.
 struct TreeParams {
   char *buf;                        // own gradient buffer (= the gradient queue)
-  char *recv[kMaxChildren];         // own receive plane for child slot s
-  char *parent_recv;                // parent's receive plane for my slot (peer); null at root
+  const char *up_src[1 + kMaxChildren];  // own buf, then each child's partial
+  char *up_dst;                     // where my partial goes (parent plane / own buf / final)
   char *child_buf[kMaxChildren];    // children's gradient buffers (peer)
   uint64_t *head_in[kMaxChildren];  // own counters written by child slot s (channel 0)
   uint64_t *head_out;               // parent's counter for my slot (peer, channel 0)
@@ -55,17 +63,20 @@ struct TreeParams {
   uint64_t *child_enq[kMaxChildren];// children's Enqueue Semaphores (peer, channel 0)
   int nchild;
   int is_root;
+  int leaf_pull;                    // leaf on a PULL edge: publishes all chunks at once
   int self_local;                   // local index of this rank (trace)
   int child_local[kMaxChildren];    // local index of each child, -1 if remote (trace)
 };
 
 enum Role { kRoleUp = 0, kRoleDown = 1 };
 
+enum { kAllChannels = -1 };  // a pulled leaf's single task covers every channel
+
 struct Task {
   int16_t local_rank;
   int16_t tree;
   int16_t role;
-  int16_t channel;
+  int16_t channel;   // kAllChannels for a pulled leaf
 };
 
 struct LaunchArgs {

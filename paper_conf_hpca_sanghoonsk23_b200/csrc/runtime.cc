@@ -169,6 +169,7 @@ struct Comm {
   int *err_host = nullptr, *err_dev = nullptr;
   std::vector<std::unique_ptr<Registration>> regs;
   std::map<std::pair<int, int>, TaskTable> tasks;  // (channels, overlap)
+  int transport = CCUBE_TRANSPORT_AUTO;
   bool sys_scope = false;
   uint64_t timeout_ns = 10000ull * 1000000ull;
   int sm_count = 0;
@@ -263,6 +264,24 @@ ccube_result_t exchange_ptrs(const std::vector<char *> &local, size_t bytes,
   return CCUBE_SUCCESS;
 }
 
+// PUSH or PULL for the edge child -> parent: PULL inside one
+// process (same GPU), PUSH across GPUs, unless forced by ccube_set_transport.
+bool edge_is_pull(int child, int parent) {
+  if (g.transport == CCUBE_TRANSPORT_PUSH) return false;
+  if (g.transport == CCUBE_TRANSPORT_PULL) return true;
+  return is_local(child) && is_local(parent);
+}
+
+bool needs_recv_planes() {
+  for (int i = 0; i < g.nlocal; ++i) {
+    const int r = g.rank0 + i;
+    for (int t = 0; t < g.ntrees; ++t)
+      for (int s = 0; s < g.trees[t].nchild[r]; ++s)
+        if (!edge_is_pull(g.trees[t].child[r][s], r)) return true;
+  }
+  return false;
+}
+
 ccube_result_t build_params(Registration *R) {
   std::vector<TreeParams> hp(static_cast<size_t>(g.nlocal) * g.ntrees);
   for (int i = 0; i < g.nlocal; ++i) {
@@ -272,8 +291,7 @@ ccube_result_t build_params(Registration *R) {
       TreeParams &p = hp[static_cast<size_t>(i) * g.ntrees + t];
       memset(&p, 0, sizeof p);
       p.buf = R->bufs[i];
-      p.recv[0] = R->recv[i];
-      p.recv[1] = R->recv[i] + R->plane;
+      p.up_src[0] = R->bufs[i];
       p.nchild = tr.nchild[r];
       p.is_root = tr.parent[r] < 0;
       p.self_local = i;
@@ -284,13 +302,22 @@ ccube_result_t build_params(Registration *R) {
       }
       p.enq = reinterpret_cast<uint64_t *>(fl + flag_offset(t, kEnq, 0));
       const int par = tr.parent[r];
-      if (par >= 0) {
+      if (par < 0) {
+        p.up_dst = R->bufs[i];  // the root's combine is final
+      } else {
         const int slot = child_slot(tr, par, r);
-        if (!R->world_recv[par] || !g.world_flags[par])
+        if (!g.world_flags[par])
           return fail(CCUBE_ERR_BOOTSTRAP, "parent %d of rank %d not mapped", par, r);
-        p.parent_recv = R->world_recv[par] + static_cast<size_t>(slot) * R->plane;
         p.head_out =
             reinterpret_cast<uint64_t *>(g.world_flags[par] + flag_offset(t, kUpHead0 + slot, 0));
+        if (edge_is_pull(r, par)) {
+          p.up_dst = R->bufs[i];  // partial stays in place; the parent reads it here
+          p.leaf_pull = tr.nchild[r] == 0;
+        } else {
+          if (!R->world_recv[par])
+            return fail(CCUBE_ERR_BOOTSTRAP, "receive plane of parent %d not mapped", par);
+          p.up_dst = R->world_recv[par] + static_cast<size_t>(slot) * R->plane;
+        }
       }
       for (int s = 0; s < tr.nchild[r]; ++s) {
         const int c = tr.child[r][s];
@@ -299,10 +326,16 @@ ccube_result_t build_params(Registration *R) {
         p.child_buf[s] = R->world_buf[c];
         p.child_enq[s] = reinterpret_cast<uint64_t *>(g.world_flags[c] + flag_offset(t, kEnq, 0));
         p.child_local[s] = is_local(c) ? c - g.rank0 : -1;
+        if (edge_is_pull(c, r)) {
+          p.up_src[1 + s] = R->world_buf[c];
+        } else {
+          if (!R->recv[i]) return fail(CCUBE_ERR_BOOTSTRAP, "receive plane missing");
+          p.up_src[1 + s] = R->recv[i] + static_cast<size_t>(s) * R->plane;
+        }
       }
     }
   }
-  CUDA_TRY(cudaMalloc(&R->d_params, sizeof(TreeParams) * hp.size()));
+  if (!R->d_params) CUDA_TRY(cudaMalloc(&R->d_params, sizeof(TreeParams) * hp.size()));
   CUDA_TRY(cudaMemcpy(R->d_params, hp.data(), sizeof(TreeParams) * hp.size(),
                       cudaMemcpyHostToDevice));
   return CCUBE_SUCCESS;
@@ -331,16 +364,23 @@ ccube_result_t do_register(void *const *bufs, size_t bytes, Registration **out) 
   R->plane = (bytes + 255) & ~static_cast<size_t>(255);
   for (int i = 0; i < g.nlocal; ++i) R->bufs.push_back(static_cast<char *>(bufs[i]));
   R->recv.assign(g.nlocal, nullptr);
-  for (int i = 0; i < g.nlocal; ++i) {
-    cudaError_t e = cudaMalloc(&R->recv[i], 2 * R->plane);
-    if (e != cudaSuccess) {
-      free_registration(R.get());
-      return fail(CCUBE_ERR_CUDA, "cudaMalloc(recv, %zu) failed: %s", 2 * R->plane,
-                  cudaGetErrorString(e));
+  // receive planes exist only for PUSH edges; multi-process communicators keep them
+  // mapped so the transport can change without another collective
+  if (g.nproc > 1 || needs_recv_planes()) {
+    for (int i = 0; i < g.nlocal; ++i) {
+      cudaError_t e = cudaMalloc(&R->recv[i], 2 * R->plane);
+      if (e != cudaSuccess) {
+        free_registration(R.get());
+        return fail(CCUBE_ERR_CUDA, "cudaMalloc(recv, %zu) failed: %s", 2 * R->plane,
+                    cudaGetErrorString(e));
+      }
     }
   }
   ccube_result_t rc = exchange_ptrs(R->bufs, bytes, &R->world_buf, &R->opened);
-  if (rc == CCUBE_SUCCESS) rc = exchange_ptrs(R->recv, 2 * R->plane, &R->world_recv, &R->opened);
+  if (rc == CCUBE_SUCCESS && R->recv[0])
+    rc = exchange_ptrs(R->recv, 2 * R->plane, &R->world_recv, &R->opened);
+  else
+    R->world_recv.assign(g.world, nullptr);
   if (rc == CCUBE_SUCCESS) rc = build_params(R.get());
   if (rc != CCUBE_SUCCESS) {
     free_registration(R.get());
@@ -374,6 +414,10 @@ ccube_result_t get_tasks(int channels, int overlap, TaskTable **out) {
     for (int t = 0; t < g.ntrees; ++t) {
       const Tree &tr = g.trees[t];
       const bool root = tr.parent[r] < 0;
+      if (!root && tr.nchild[r] == 0 && edge_is_pull(r, tr.parent[r])) {
+        ts.push_back(Task{(int16_t)i, (int16_t)t, (int16_t)kRoleUp, (int16_t)kAllChannels});
+        continue;
+      }
       const bool down = tr.nchild[r] > 0 && (!root || !overlap);
       for (int j = 0; j < channels; ++j)
         ts.push_back(Task{(int16_t)i, (int16_t)t, (int16_t)kRoleUp, (int16_t)j});
@@ -449,10 +493,11 @@ ccube_result_t allreduce_impl(void *const *bufs, size_t count, ccube_dtype_t dty
   a.tasks = tt->d_tasks;
 
   // all CTAs spin on each other: they must be co-resident
-  auto key = std::make_pair((int)dtype, g.threads);
+  const int cta_threads = g.threads + 32;  // data warps + the control warp
+  auto key = std::make_pair((int)dtype, cta_threads);
   if (!g.max_blocks.count(key)) {
     int b = 0;
-    const int rc = query_max_blocks_per_sm(dtype, g.sys_scope, g.threads, &b);
+    const int rc = query_max_blocks_per_sm(dtype, g.sys_scope, cta_threads, &b);
     if (rc != cudaSuccess)
       return fail(CCUBE_ERR_CUDA, "occupancy query failed: %s",
                   cudaGetErrorString(static_cast<cudaError_t>(rc)));
@@ -464,7 +509,7 @@ ccube_result_t allreduce_impl(void *const *bufs, size_t count, ccube_dtype_t dty
                 "%d CTAs (channels=%d) cannot be co-resident (capacity %d); lower channels",
                 tt->n, g.channels, cap);
 
-  const int rc = launch_tree_allreduce(a, dtype, g.sys_scope, tt->n, g.threads, stream);
+  const int rc = launch_tree_allreduce(a, dtype, g.sys_scope, tt->n, cta_threads, stream);
   if (rc != cudaSuccess)
     return fail(CCUBE_ERR_CUDA, "kernel launch failed: %s",
                 cudaGetErrorString(static_cast<cudaError_t>(rc)));
@@ -588,8 +633,11 @@ ccube_result_t ccube_init(const ccube_world_t *world, ccube_tree_kind_t tree_kin
     return fail(CCUBE_ERR_INVALID_ARG, "CCUBE_CHANNELS %d out of range", channels);
   CC_TRY(check_chunk_channels(chunk_bytes, channels));
   int threads = env_int("CCUBE_THREADS", 512);
-  if (threads < 64 || threads > 512 || threads % 32)
-    return fail(CCUBE_ERR_INVALID_ARG, "CCUBE_THREADS %d out of range [64, 512]", threads);
+  if (threads < 32 || threads > 512 || threads % 32)
+    return fail(CCUBE_ERR_INVALID_ARG, "CCUBE_THREADS %d out of range [32, 512]", threads);
+  const int transport = env_int("CCUBE_TRANSPORT", CCUBE_TRANSPORT_AUTO);
+  if (transport < CCUBE_TRANSPORT_AUTO || transport > CCUBE_TRANSPORT_PULL)
+    return fail(CCUBE_ERR_INVALID_ARG, "CCUBE_TRANSPORT %d out of range", transport);
 
   g = Comm();
   g.world = P;
@@ -604,6 +652,7 @@ ccube_result_t ccube_init(const ccube_world_t *world, ccube_tree_kind_t tree_kin
   g.chunk_bytes = chunk_bytes;
   g.channels = channels;
   g.threads = threads;
+  g.transport = transport;
   g.overlap = 1;
   g.sys_scope = g.nproc > 1;
   g.timeout_ns = static_cast<uint64_t>(env_int("CCUBE_WATCHDOG_MS", 10000)) * 1000000ull;
@@ -782,10 +831,31 @@ ccube_result_t ccube_set_channels(int channels) {
 ccube_result_t ccube_set_threads(int threads) {
   std::lock_guard<std::mutex> lk(g_mu);
   if (!g.init) return fail(CCUBE_ERR_NOT_INITIALIZED, "ccube_init has not been called");
-  if (threads < 64 || threads > 512 || threads % 32)
-    return fail(CCUBE_ERR_INVALID_ARG, "threads %d out of range [64, 512] (multiple of 32)",
+  if (threads < 32 || threads > 512 || threads % 32)
+    return fail(CCUBE_ERR_INVALID_ARG, "threads %d out of range [32, 512] (multiple of 32)",
                 threads);
   g.threads = threads;
+  return CCUBE_SUCCESS;
+}
+
+ccube_result_t ccube_set_transport(int mode) {
+  std::lock_guard<std::mutex> lk(g_mu);
+  if (!g.init) return fail(CCUBE_ERR_NOT_INITIALIZED, "ccube_init has not been called");
+  if (mode < CCUBE_TRANSPORT_AUTO || mode > CCUBE_TRANSPORT_PULL)
+    return fail(CCUBE_ERR_INVALID_ARG, "transport %d out of range", mode);
+  if (mode == g.transport) return CCUBE_SUCCESS;
+  CUDA_TRY(cudaDeviceSynchronize());
+  g.transport = mode;
+  for (auto &kv : g.tasks) cudaFree(kv.second.d_tasks);
+  g.tasks.clear();
+  for (auto &R : g.regs) {
+    if (!R->recv[0] && needs_recv_planes()) {  // loopback only: planes are local
+      for (int i = 0; i < g.nlocal; ++i) CUDA_TRY(cudaMalloc(&R->recv[i], 2 * R->plane));
+      R->world_recv.assign(g.world, nullptr);
+      for (int i = 0; i < g.nlocal; ++i) R->world_recv[g.rank0 + i] = R->recv[i];
+    }
+    CC_TRY(build_params(R.get()));
+  }
   return CCUBE_SUCCESS;
 }
 
@@ -827,6 +897,7 @@ ccube_result_t ccube_get_info(ccube_info_t *info) {
   info->channels = g.channels;
   info->threads = g.threads;
   info->overlap = g.overlap;
+  info->transport = g.transport;
   info->chunk_bytes = g.chunk_bytes;
   info->epoch_base[0] = g.base[0];
   info->epoch_base[1] = g.base[1];

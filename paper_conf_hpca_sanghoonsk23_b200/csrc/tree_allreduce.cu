@@ -5,26 +5,28 @@
 // `tree` and walks the tree-local chunks k = 0..K_t-1 in order (the tree keeps
 // chunk order, Obs #3 P:L145; the gradient queue relies on it).
 //
-//   role UP   (a4, reduce-up): wait until each child's partial of chunk k
-//             sits in my receive plane, combine own ⊕ child_lo ⊕ child_hi in that
-//             fixed order (R2/R3) and push the result with 128-bit stores into the
-//             parent's receive plane (NVLink peer memory), then release the
-//             parent's head counter.  The root instead writes the final value into
-//             its own buffer and — in C1 — straight into its children's
+//   role UP   (a4, reduce-up): once every child's partial of chunk k is
+//             available, combine own ⊕ child_lo ⊕ child_hi in that fixed order
+//             (R2/R3) and hand the result to the parent (PUSH: 128-bit stores into
+//             the parent's receive plane over NVLink; PULL: in place in my own
+//             buffer, read by the parent).  The root writes the final value into its
+//             own buffer and — in C1 — straight into its children's
 //             buffers, publishing their Enqueue Semaphores: the reduce->broadcast
 //             turnaround costs no extra pass.
-//   role DOWN (a5, broadcast-down): wait on my own Enqueue Semaphore (written by
-//             my parent after it stored chunk k into my buffer, Fig 9), copy
-//             chunk k from my buffer into each child's buffer and publish the
-//             children's semaphores.  In B mode the root also runs a DOWN task that
-//             starts only after all K_t chunks are reduced (Fig 7(a)).
-// Leaves have no DOWN task; their UP task finally waits until the whole buffer
-// has landed so that the kernel completes only when the result is final.
+//   role DOWN (a5, broadcast-down): once my Enqueue Semaphore says chunk k landed
+//             in my buffer (written there by my parent, Fig 9), copy it into
+//             each child's buffer and publish the children's semaphores.  In B mode
+//             the root also runs a DOWN task that starts only after all K_t chunks
+//             are reduced (Fig 7(a)).
 //
-// Synchronisation (a7, replacing Fig 11's atomicCAS locks): single-writer
-// monotone u64 counters; producer = CTA barrier + fence.acq_rel + relaxed store,
-// consumer = one thread's acquire load + CTA barrier.  .sys scope when peers are
-// other GPUs, .gpu scope in loopback.  Every spin has a %globaltimer watchdog.
+// CTA = 1 control warp + W data warps (warp specialisation).  The control warp
+// polls the upstream counters (one lane per child, .gpu/.sys acquire), publishes
+// "chunks ready" to the data warps through shared memory, collects per-warp
+// "chunks done" counters and releases the downstream counters (fence + one relaxed
+// store covering every chunk finished so far: counters are monotone and waits are
+// ">=", Fig 11 "check").  Data warps never wait on a fence; each streams its share
+// of every chunk slice with 128-bit accesses, U vectors in flight per source.
+// Every spin has a %globaltimer watchdog (CCUBE_WATCHDOG_MS).
 #include <cuda_bf16.h>
 #include <cuda_runtime.h>
 #include <stdint.h>
@@ -35,7 +37,8 @@ namespace ccube {
 namespace {
 
 constexpr int kUnroll = 4;
-constexpr int kMaxThreads = 512;
+constexpr int kMaxThreads = 544;  // 16 data warps + the control warp
+constexpr int kMaxDataWarps = 16;
 
 __device__ __forceinline__ uint64_t globaltimer() {
   uint64_t t;
@@ -69,39 +72,68 @@ __device__ __forceinline__ void st_relaxed(uint64_t *p, uint64_t v) {
     asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
 
-// Spin until *p >= target.  Returns false if the watchdog fired or another CTA
-// already reported an error (then the caller must leave the kernel).
-template <bool SYS>
-__device__ bool wait_geq(const uint64_t *p, uint64_t target, int *err, uint64_t timeout_ns,
-                         uint64_t *seen) {
-  uint64_t v = ld_acquire<SYS>(p);
-  if (v >= target) {
-    *seen = v;
-    return true;
+// CTA-scope release/acquire on shared memory (control <-> data warps)
+__device__ __forceinline__ void st_release_cta(uint64_t *p, uint64_t v) {
+  asm volatile("st.release.cta.shared.u64 [%0], %1;" ::"r"((uint32_t)__cvta_generic_to_shared(p)),
+               "l"(v)
+               : "memory");
+}
+__device__ __forceinline__ uint64_t ld_acquire_cta(const uint64_t *p) {
+  uint64_t v;
+  asm volatile("ld.acquire.cta.shared.u64 %0, [%1];"
+               : "=l"(v)
+               : "r"((uint32_t)__cvta_generic_to_shared(p))
+               : "memory");
+  return v;
+}
+
+__device__ __forceinline__ uint64_t warp_min(uint64_t v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    const uint64_t w = __shfl_xor_sync(0xffffffffu, v, o);
+    v = w < v ? w : v;
   }
-  const uint64_t t0 = globaltimer();
-  uint64_t next_check = t0 + 1000000ull;  // look at the error word once per ms
-  while (true) {
-    v = ld_acquire<SYS>(p);
-    if (v >= target) {
-      *seen = v;
-      return true;
-    }
-    const uint64_t now = globaltimer();
-    if (now >= next_check) {
-      if (*reinterpret_cast<volatile int *>(err) != 0) return false;
-      if (now - t0 > timeout_ns) {
-        reinterpret_cast<volatile int *>(err)[1] = static_cast<int>(blockIdx.x);
-        reinterpret_cast<volatile int *>(err)[2] = static_cast<int>(target & 0x7fffffff);
-        reinterpret_cast<volatile int *>(err)[3] = static_cast<int>(v & 0x7fffffff);
-        __threadfence_system();
-        *reinterpret_cast<volatile int *>(err) = 1;  // 1 = watchdog timeout
-        __threadfence_system();
-        return false;
-      }
-      next_check = now + 1000000ull;
-    }
+  return v;
+}
+
+struct Shared {
+  uint64_t ready;                 // chunks whose inputs are available (control -> data)
+  uint64_t done[kMaxDataWarps];   // chunks finished by data warp w (data -> control)
+  int abort;
+};
+
+// Watchdog bookkeeping for the control warp.
+struct Watch {
+  uint64_t last;       // time of the last progress
+  uint64_t next_err;   // next time to look at the host error word
+  uint32_t spins;
+};
+
+__device__ __forceinline__ void watch_reset(Watch &w) {
+  w.last = globaltimer();
+  w.next_err = w.last + 1000000ull;
+  w.spins = 0;
+}
+
+// true = keep going; false = abort (timeout here or error elsewhere)
+__device__ __forceinline__ bool watch_tick(Watch &w, const LaunchArgs &a, uint64_t target,
+                                           uint64_t seen) {
+  if (++w.spins & 63) return true;
+  const uint64_t now = globaltimer();
+  if (now < w.next_err) return true;
+  w.next_err = now + 1000000ull;
+  if (*reinterpret_cast<volatile int *>(a.err) != 0) return false;
+  if (now - w.last > a.timeout_ns) {
+    volatile int *e = reinterpret_cast<volatile int *>(a.err);
+    e[1] = static_cast<int>(blockIdx.x);
+    e[2] = static_cast<int>(target & 0x7fffffff);
+    e[3] = static_cast<int>(seen & 0x7fffffff);
+    __threadfence_system();
+    e[0] = 1;  // 1 = watchdog timeout
+    __threadfence_system();
+    return false;
   }
+  return true;
 }
 
 // ---- element combine (R2/R3) ------------------------------------------------
@@ -163,9 +195,11 @@ struct Combine<kFloat32> {
 template <>
 struct Combine<kBFloat16> {
   // widen to fp32, add in the fixed order, round ONCE per node output (RNE)
-  __device__ __forceinline__ static uint32_t word(const uint32_t *w, int n) {
+  template <int N>
+  __device__ __forceinline__ static uint32_t word(const uint32_t (&w)[N]) {
     float lo = bf_lo(w[0]), hi = bf_hi(w[0]);
-    for (int i = 1; i < n; ++i) {
+#pragma unroll
+    for (int i = 1; i < N; ++i) {
       lo = __fadd_rn(lo, bf_lo(w[i]));
       hi = __fadd_rn(hi, bf_hi(w[i]));
     }
@@ -173,11 +207,14 @@ struct Combine<kBFloat16> {
   }
   template <int N>
   __device__ __forceinline__ static uint4 vec(const uint4 (&v)[N]) {
-    if (N == 1) return v[0];  // a leaf forwards its own bits untouched
-    uint32_t a[N], b[N], c[N], d[N];
+    if constexpr (N == 1) {
+      return v[0];  // a leaf forwards its own bits untouched
+    } else {
+      uint32_t a[N], b[N], c[N], d[N];
 #pragma unroll
-    for (int i = 0; i < N; ++i) { a[i] = v[i].x; b[i] = v[i].y; c[i] = v[i].z; d[i] = v[i].w; }
-    return make_uint4(word(a, N), word(b, N), word(c, N), word(d, N));
+      for (int i = 0; i < N; ++i) { a[i] = v[i].x; b[i] = v[i].y; c[i] = v[i].z; d[i] = v[i].w; }
+      return make_uint4(word<N>(a), word<N>(b), word<N>(c), word<N>(d));
+    }
   }
   template <int N>
   __device__ __forceinline__ static void scalar(const char *const *src, char *const *dst,
@@ -196,40 +233,40 @@ struct Combine<kBFloat16> {
   }
 };
 
-// Combine NIN sources element-wise over elements [elo, ehi) and store to NOUT
-// destinations.  Sources are local HBM (own buffer / own receive planes);
-// destinations may be peer memory.  128-bit accesses, kUnroll vectors in flight
-// per thread per source, then the scalar tail of a ragged last chunk.
+// One data warp's share of elements [elo, ehi): vectors w*32+lane, stepping W*32,
+// U vectors per source in flight; the ragged scalar tail goes to warp 0.
+// Sources are local HBM or (PULL) peer buffers; destinations may be peer memory.
 template <int DT, int NIN, int NOUT>
-__device__ __forceinline__ void process(const char *const *src, char *const *dst, uint64_t elo,
-                                        uint64_t ehi) {
+__device__ __forceinline__ void process_warp(const char *const *src, char *const *dst,
+                                             uint64_t elo, uint64_t ehi, int w, int W) {
   constexpr int ES = DT == kBFloat16 ? 2 : 4;
   constexpr int VE = 16 / ES;
   if (ehi <= elo) return;
   const uint64_t n = ehi - elo;
   const uint64_t nv = n / VE;
+  const int lane = threadIdx.x & 31;
   const uint4 *s[NIN];
   uint4 *d[NOUT];
 #pragma unroll
   for (int i = 0; i < NIN; ++i) s[i] = reinterpret_cast<const uint4 *>(src[i] + elo * ES);
 #pragma unroll
   for (int i = 0; i < NOUT; ++i) d[i] = reinterpret_cast<uint4 *>(dst[i] + elo * ES);
-  const uint64_t nt = blockDim.x;
-  uint64_t i = threadIdx.x;
-  for (; i + (kUnroll - 1) * nt < nv; i += kUnroll * nt) {
+  const uint64_t step = static_cast<uint64_t>(W) * 32;
+  uint64_t i = static_cast<uint64_t>(w) * 32 + lane;
+  for (; i + (kUnroll - 1) * step < nv; i += kUnroll * step) {
     uint4 v[kUnroll][NIN];
 #pragma unroll
     for (int u = 0; u < kUnroll; ++u)
 #pragma unroll
-      for (int q = 0; q < NIN; ++q) v[u][q] = __ldcg(s[q] + i + u * nt);
+      for (int q = 0; q < NIN; ++q) v[u][q] = __ldcg(s[q] + i + u * step);
 #pragma unroll
     for (int u = 0; u < kUnroll; ++u) {
       const uint4 r = Combine<DT>::template vec<NIN>(v[u]);
 #pragma unroll
-      for (int q = 0; q < NOUT; ++q) d[q][i + u * nt] = r;
+      for (int q = 0; q < NOUT; ++q) d[q][i + u * step] = r;
     }
   }
-  for (; i < nv; i += nt) {
+  for (; i < nv; i += step) {
     uint4 v[NIN];
 #pragma unroll
     for (int q = 0; q < NIN; ++q) v[q] = __ldcg(s[q] + i);
@@ -237,34 +274,36 @@ __device__ __forceinline__ void process(const char *const *src, char *const *dst
 #pragma unroll
     for (int q = 0; q < NOUT; ++q) d[q][i] = r;
   }
-  const char *ss[NIN];
-  char *dd[NOUT];
+  if (w == 0) {
+    const char *ss[NIN];
+    char *dd[NOUT];
 #pragma unroll
-  for (int q = 0; q < NIN; ++q) ss[q] = src[q] + elo * ES;
+    for (int q = 0; q < NIN; ++q) ss[q] = src[q] + elo * ES;
 #pragma unroll
-  for (int q = 0; q < NOUT; ++q) dd[q] = dst[q] + elo * ES;
-  for (uint64_t e = nv * VE + threadIdx.x; e < n; e += nt)
-    Combine<DT>::template scalar<NIN>(ss, dd, NOUT, e);
+    for (int q = 0; q < NOUT; ++q) dd[q] = dst[q] + elo * ES;
+    for (uint64_t e = nv * VE + lane; e < n; e += 32)
+      Combine<DT>::template scalar<NIN>(ss, dd, NOUT, e);
+  }
 }
 
 template <int DT, int NIN>
 __device__ __forceinline__ void process_nout(const char *const *src, char *const *dst, int nout,
-                                             uint64_t elo, uint64_t ehi) {
+                                             uint64_t elo, uint64_t ehi, int w, int W) {
   switch (nout) {
-    case 1: process<DT, NIN, 1>(src, dst, elo, ehi); break;
-    case 2: process<DT, NIN, 2>(src, dst, elo, ehi); break;
-    case 3: process<DT, NIN, 3>(src, dst, elo, ehi); break;
+    case 1: process_warp<DT, NIN, 1>(src, dst, elo, ehi, w, W); break;
+    case 2: process_warp<DT, NIN, 2>(src, dst, elo, ehi, w, W); break;
+    case 3: process_warp<DT, NIN, 3>(src, dst, elo, ehi, w, W); break;
     default: break;
   }
 }
 
 template <int DT>
 __device__ __forceinline__ void dispatch(const char *const *src, int nin, char *const *dst,
-                                         int nout, uint64_t elo, uint64_t ehi) {
+                                         int nout, uint64_t elo, uint64_t ehi, int w, int W) {
   switch (nin) {
-    case 1: process_nout<DT, 1>(src, dst, nout, elo, ehi); break;
-    case 2: process_nout<DT, 2>(src, dst, nout, elo, ehi); break;
-    case 3: process_nout<DT, 3>(src, dst, nout, elo, ehi); break;
+    case 1: process_nout<DT, 1>(src, dst, nout, elo, ehi, w, W); break;
+    case 2: process_nout<DT, 2>(src, dst, nout, elo, ehi, w, W); break;
+    case 3: process_nout<DT, 3>(src, dst, nout, elo, ehi, w, W); break;
     default: break;
   }
 }
@@ -279,130 +318,192 @@ __device__ __forceinline__ void slice_range(const LaunchArgs &a, int t, int j, u
   *hi = h > l ? h : l;
 }
 
-__device__ __forceinline__ void trace_landing(const LaunchArgs &a, int local, int t, uint32_t k,
-                                              int j) {
-  if (a.trace == nullptr || local < 0 || k >= a.trace_kmax) return;
-  const uint64_t idx =
-      ((static_cast<uint64_t>(local) * a.ntrees + t) * a.trace_kmax + k) * a.nchannels + j;
-  a.trace[idx] = globaltimer();
+__device__ __forceinline__ void trace_landing(const LaunchArgs &a, int local, int t, uint32_t k0,
+                                              uint32_t k1, int j) {
+  if (a.trace == nullptr || local < 0) return;
+  const uint64_t now = globaltimer();
+  for (uint32_t k = k0; k < k1 && k < a.trace_kmax; ++k) {
+    const uint64_t idx =
+        ((static_cast<uint64_t>(local) * a.ntrees + t) * a.trace_kmax + k) * a.nchannels + j;
+    a.trace[idx] = now;
+  }
 }
 
-template <int DT, bool SYS>
-__device__ void up_role(const LaunchArgs &a, const TreeParams &p, int t, int j, int *sh_ok) {
+// ---- control warp --------------------------------------------------------------
+// Releases chunks [pub, d) downstream: one fence, then one store per counter.
+template <bool SYS>
+__device__ __forceinline__ void publish(const LaunchArgs &a, const TreeParams &p, int role, int t,
+                                        int j, uint32_t pub, uint32_t d, uint64_t base) {
+  const int stride = j * kFlagStrideU64;
+  const uint64_t v = base + d;
+  fence_release<SYS>();
+  if (role == kRoleUp && !p.is_root) {
+    st_relaxed<SYS>(p.head_out + stride, v);
+    return;
+  }
+  if (role == kRoleUp) {  // root: the chunk is final in my own buffer
+    st_relaxed<SYS>(p.enq + stride, v);
+    trace_landing(a, p.self_local, t, pub, d, j);
+    if (!a.overlap) return;
+  }
+  for (int s = 0; s < p.nchild; ++s) {  // root in C1, or any DOWN task
+    st_relaxed<SYS>(p.child_enq[s] + stride, v);
+    trace_landing(a, p.child_local[s], t, pub, d, j);
+  }
+}
+
+template <bool SYS>
+__device__ void control_warp(const LaunchArgs &a, const TreeParams &p, int role, int t, int j,
+                             int W, Shared &sh) {
+  const int lane = threadIdx.x & 31;
   const uint32_t K = a.K[t];
   const uint64_t base = a.base[t];
   const int stride = j * kFlagStrideU64;
-  uint64_t ready = 0;  // thread 0: tree-local chunks known complete at every child
-  const char *src[3] = {p.buf, p.recv[0], p.recv[1]};
+  // upstream counters: UP waits on each child's head, DOWN on my own semaphore
+  const uint64_t *up = nullptr;
+  if (role == kRoleUp) {
+    if (lane < p.nchild) up = p.head_in[lane] + stride;
+  } else if (lane == 0) {
+    up = p.enq + stride;
+  }
+  const bool hold_all = role == kRoleDown && p.is_root;  // B-mode root (Obs #1)
+  uint64_t ready = (role == kRoleUp && p.nchild == 0) ? K : 0;  // a leaf's input is ready
+  if (lane == 0) st_release_cta(&sh.ready, ready);
+  uint32_t pub = 0;
+  Watch wd;
+  watch_reset(wd);
+  while (pub < K) {
+    bool moved = false;
+    if (ready < K) {
+      uint64_t v = up ? ld_acquire<SYS>(up) : ~0ull;
+      v = warp_min(v);
+      uint64_t r = v > base ? v - base : 0;
+      if (r > K) r = K;
+      if (hold_all && r < K) r = 0;
+      if (r > ready) {
+        ready = r;
+        if (lane == 0) st_release_cta(&sh.ready, ready);
+        moved = true;
+      }
+    }
+    uint64_t d = lane < W ? ld_acquire_cta(&sh.done[lane]) : ~0ull;
+    d = warp_min(d);
+    if (d > pub) {
+      __syncwarp();
+      if (lane == 0) publish<SYS>(a, p, role, t, j, pub, static_cast<uint32_t>(d), base);
+      pub = static_cast<uint32_t>(d);
+      moved = true;
+    }
+    if (moved) {
+      watch_reset(wd);
+    } else if (!watch_tick(wd, a, base + ready + 1, base + pub)) {
+      if (lane == 0) {
+        *reinterpret_cast<volatile int *>(&sh.abort) = 1;
+        st_relaxed<SYS>(p.enq + stride, ~0ull);  // release gradient-queue waiters
+      }
+      return;
+    }
+  }
+  // a leaf's kernel completes only once the whole result has landed in its buffer
+  if (role == kRoleUp && !p.is_root && p.nchild == 0 && lane == 0) {
+    watch_reset(wd);
+    while (ld_acquire<SYS>(p.enq + stride) < base + K) {
+      if (!watch_tick(wd, a, base + K, 0)) {
+        st_relaxed<SYS>(p.enq + stride, ~0ull);
+        return;
+      }
+    }
+  }
+}
+
+// A leaf on a PULL edge: its input already sits where the parent reads it.  One
+// warp publishes every channel's head at once and waits for the result.
+template <bool SYS>
+__device__ void pulled_leaf(const LaunchArgs &a, const TreeParams &p, int t) {
+  const int lane = threadIdx.x & 31;
+  const uint32_t K = a.K[t];
+  const uint64_t base = a.base[t];
+  fence_release<SYS>();
+  for (int j = lane; j < static_cast<int>(a.nchannels); j += 32)
+    st_relaxed<SYS>(p.head_out + j * kFlagStrideU64, base + K);
+  for (int j = lane; j < static_cast<int>(a.nchannels); j += 32) {
+    Watch wd;
+    watch_reset(wd);
+    while (ld_acquire<SYS>(p.enq + j * kFlagStrideU64) < base + K) {
+      if (!watch_tick(wd, a, base + K, 0)) {
+        st_relaxed<SYS>(p.enq + j * kFlagStrideU64, ~0ull);
+        break;
+      }
+    }
+  }
+}
+
+// ---- data warps ----------------------------------------------------------------
+template <int DT>
+__device__ void data_warp(const LaunchArgs &a, const TreeParams &p, int role, int t, int j,
+                          int w, int W, Shared &sh) {
+  const int lane = threadIdx.x & 31;
+  const uint32_t K = a.K[t];
+  const char *src[3];
   char *dst[3];
-  int nout = 1;
-  if (p.is_root) {
-    dst[0] = p.buf;
-    if (a.overlap) {
+  int nin, nout;
+  if (role == kRoleUp) {
+    nin = 1 + p.nchild;
+    for (int q = 0; q < nin; ++q) src[q] = p.up_src[q];
+    dst[0] = p.up_dst;
+    nout = 1;
+    if (p.is_root && a.overlap) {  // C1 turnaround: final straight into the children
       for (int s = 0; s < p.nchild; ++s) dst[1 + s] = p.child_buf[s];
       nout += p.nchild;
     }
   } else {
-    dst[0] = p.parent_recv;
+    nin = 1;
+    src[0] = p.buf;
+    for (int s = 0; s < p.nchild; ++s) dst[s] = p.child_buf[s];
+    nout = p.nchild;
   }
-  const int nin = 1 + p.nchild;
-  for (uint32_t k = 0; k < K; ++k) {
-    if (threadIdx.x == 0) {
-      int ok = 1;
-      if (p.nchild > 0 && ready <= k) {
-        uint64_t m = ~0ull;
-        for (int s = 0; s < p.nchild && ok; ++s) {
-          uint64_t seen = 0;
-          ok = wait_geq<SYS>(p.head_in[s] + stride, base + k + 1, a.err, a.timeout_ns, &seen);
-          m = seen < m ? seen : m;
-        }
-        ready = m - base;
-      }
-      *sh_ok = ok;
-    }
-    __syncthreads();
-    if (!*sh_ok) {
-      if (threadIdx.x == 0) st_relaxed<SYS>(p.enq + stride, ~0ull);  // release gradq waiters
-      return;
-    }
-    uint64_t lo, hi;
-    slice_range(a, t, j, k, &lo, &hi);
-    dispatch<DT>(src, nin, dst, nout, lo, hi);
-    __syncthreads();  // every store of chunk k issued (and ordered) before the release
-    if (threadIdx.x == 0) {
-      const uint64_t v = base + k + 1;
-      fence_release<SYS>();
-      if (p.is_root) {
-        st_relaxed<SYS>(p.enq + stride, v);
-        trace_landing(a, p.self_local, t, k, j);
-        if (a.overlap) {
-          for (int s = 0; s < p.nchild; ++s) {
-            st_relaxed<SYS>(p.child_enq[s] + stride, v);
-            trace_landing(a, p.child_local[s], t, k, j);
-          }
-        }
-      } else {
-        st_relaxed<SYS>(p.head_out + stride, v);
-      }
-    }
-  }
-  if (!p.is_root && p.nchild == 0 && threadIdx.x == 0) {
-    // leaf: the kernel may complete only once the whole result has landed here
-    uint64_t seen;
-    if (!wait_geq<SYS>(p.enq + stride, base + K, a.err, a.timeout_ns, &seen))
-      st_relaxed<SYS>(p.enq + stride, ~0ull);
-  }
-}
-
-template <int DT, bool SYS>
-__device__ void down_role(const LaunchArgs &a, const TreeParams &p, int t, int j, int *sh_ok) {
-  const uint32_t K = a.K[t];
-  const uint64_t base = a.base[t];
-  const int stride = j * kFlagStrideU64;
   uint64_t ready = 0;
-  const char *src[1] = {p.buf};
-  char *dst[2] = {p.child_buf[0], p.child_buf[1]};
   for (uint32_t k = 0; k < K; ++k) {
-    if (threadIdx.x == 0) {
-      int ok = 1;
-      if (ready <= k) {
-        // B mode root: hold every chunk until the whole reduction is done (Obs #1)
-        const uint64_t target = p.is_root ? base + K : base + k + 1;
-        uint64_t seen = 0;
-        ok = wait_geq<SYS>(p.enq + stride, target, a.err, a.timeout_ns, &seen);
-        ready = seen - base;
+    if (ready <= k) {
+      uint64_t r = 0;
+      if (lane == 0) {
+        do {
+          r = ld_acquire_cta(&sh.ready);
+        } while (r <= k && !*reinterpret_cast<volatile int *>(&sh.abort));
       }
-      *sh_ok = ok;
-    }
-    __syncthreads();
-    if (!*sh_ok) {
-      if (threadIdx.x == 0) st_relaxed<SYS>(p.enq + stride, ~0ull);  // release gradq waiters
-      return;
+      r = __shfl_sync(0xffffffffu, r, 0);
+      if (r <= k) return;  // aborted
+      ready = r;
     }
     uint64_t lo, hi;
     slice_range(a, t, j, k, &lo, &hi);
-    dispatch<DT>(src, 1, dst, p.nchild, lo, hi);
-    __syncthreads();
-    if (threadIdx.x == 0) {
-      const uint64_t v = base + k + 1;
-      fence_release<SYS>();
-      for (int s = 0; s < p.nchild; ++s) {
-        st_relaxed<SYS>(p.child_enq[s] + stride, v);
-        trace_landing(a, p.child_local[s], t, k, j);
-      }
-    }
+    dispatch<DT>(src, nin, dst, nout, lo, hi, w, W);
+    __syncwarp();
+    if (lane == 0) st_release_cta(&sh.done[w], k + 1);
   }
 }
 
 template <int DT, bool SYS>
 __global__ void __launch_bounds__(kMaxThreads) tree_allreduce_kernel(const LaunchArgs a) {
-  __shared__ int sh_ok;
+  __shared__ Shared sh;
   const Task task = a.tasks[blockIdx.x];
   const TreeParams &p = a.params[task.local_rank * a.ntrees + task.tree];
-  if (task.role == kRoleUp)
-    up_role<DT, SYS>(a, p, task.tree, task.channel, &sh_ok);
+  const int warp = threadIdx.x >> 5;
+  if (task.channel == kAllChannels) {
+    if (warp == 0) pulled_leaf<SYS>(a, p, task.tree);
+    return;
+  }
+  const int W = (blockDim.x >> 5) - 1;
+  if (threadIdx.x == 0) {
+    sh.ready = 0;
+    sh.abort = 0;
+  }
+  if (threadIdx.x < kMaxDataWarps) sh.done[threadIdx.x] = 0;
+  __syncthreads();
+  if (warp == 0)
+    control_warp<SYS>(a, p, task.role, task.tree, task.channel, W, sh);
   else
-    down_role<DT, SYS>(a, p, task.tree, task.channel, &sh_ok);
+    data_warp<DT>(a, p, task.role, task.tree, task.channel, warp - 1, W, sh);
 }
 
 struct GateArgs {
@@ -418,8 +519,14 @@ struct GateArgs {
 template <bool SYS>
 __global__ void gate_kernel(const GateArgs g) {
   for (int i = threadIdx.x; i < g.n; i += blockDim.x) {
-    uint64_t seen;
-    wait_geq<SYS>(g.ctr[i], g.target[i], g.err, g.timeout_ns, &seen);
+    const uint64_t t0 = globaltimer();
+    while (ld_acquire<SYS>(g.ctr[i]) < g.target[i]) {
+      if (globaltimer() - t0 > g.timeout_ns) {
+        *reinterpret_cast<volatile int *>(g.err) = 2;  // 2 = gate timeout
+        __threadfence_system();
+        break;
+      }
+    }
   }
 }
 
@@ -429,11 +536,18 @@ int launch_t(const LaunchArgs &a, int grid, int threads, cudaStream_t s) {
   return static_cast<int>(cudaGetLastError());
 }
 
+template <int DT, bool SYS>
+const void *kernel_ptr() {
+  return reinterpret_cast<const void *>(tree_allreduce_kernel<DT, SYS>);
+}
+
 }  // namespace
 
 int launch_tree_allreduce(const LaunchArgs &args, int dtype, bool sys_scope, int grid,
                           int threads, void *stream) {
-  if (threads > kMaxThreads || threads < 32 || threads % 32) return cudaErrorInvalidValue;
+  if (threads > kMaxThreads || threads < 64 || threads % 32 ||
+      threads / 32 - 1 > kMaxDataWarps)
+    return cudaErrorInvalidValue;
   cudaStream_t s = static_cast<cudaStream_t>(stream);
   switch (dtype) {
     case kInt32:
@@ -474,16 +588,13 @@ int query_max_blocks_per_sm(int dtype, bool sys_scope, int threads, int *blocks)
   const void *fn = nullptr;
   switch (dtype) {
     case kInt32:
-      fn = sys_scope ? (const void *)tree_allreduce_kernel<kInt32, true>
-                     : (const void *)tree_allreduce_kernel<kInt32, false>;
+      fn = sys_scope ? kernel_ptr<kInt32, true>() : kernel_ptr<kInt32, false>();
       break;
     case kFloat32:
-      fn = sys_scope ? (const void *)tree_allreduce_kernel<kFloat32, true>
-                     : (const void *)tree_allreduce_kernel<kFloat32, false>;
+      fn = sys_scope ? kernel_ptr<kFloat32, true>() : kernel_ptr<kFloat32, false>();
       break;
     default:
-      fn = sys_scope ? (const void *)tree_allreduce_kernel<kBFloat16, true>
-                     : (const void *)tree_allreduce_kernel<kBFloat16, false>;
+      fn = sys_scope ? kernel_ptr<kBFloat16, true>() : kernel_ptr<kBFloat16, false>();
       break;
   }
   return static_cast<int>(cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks, fn, threads, 0));

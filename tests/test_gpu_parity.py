@@ -23,9 +23,12 @@ def comm():
     """Yields an init function; always finalizes."""
     state = {"on": False}
 
-    def _init(P, kind="single", chunk_bytes=4096, channels=None, overlap=True, threads=None):
+    def _init(P, kind="single", chunk_bytes=4096, channels=None, overlap=True, threads=None,
+              transport=None):
         ccube.init_loopback(P, kind, chunk_bytes)
         state["on"] = True
+        if transport is not None:
+            ccube.set_transport(transport)
         if channels is not None:
             ccube.set_channels(channels)
         if threads is not None:
@@ -49,10 +52,12 @@ def _run(P, kind, dtype, count, chunk_bytes, seed=5):
 @pytest.mark.parametrize("kind", ["single", "double"])
 @pytest.mark.parametrize("dtype", ["int32", "float32", "bfloat16"])
 @pytest.mark.parametrize("overlap", [True, False])
-def test_parity_small(comm, P, kind, dtype, overlap):
-    """Several chunks (K = 8), 4 channels, ragged tail (not a whole vector)."""
+@pytest.mark.parametrize("transport", ["pull", "push"])
+def test_parity_small(comm, P, kind, dtype, overlap, transport):
+    """Several chunks (K = 8), 4 channels, ragged tail (not a whole vector); both edge
+    transports (PUSH = the cross-GPU path, PULL = the same-GPU path)."""
     chunk = 4096
-    comm(P, kind, chunk, channels=4, overlap=overlap)
+    comm(P, kind, chunk, channels=4, overlap=overlap, transport=transport)
     E = chunk // arith.ELEM_SIZE[dtype]
     count = 7 * E + 13
     xs, outs = _run(P, kind, dtype, count, chunk)
@@ -72,7 +77,7 @@ def test_parity_channels(comm, channels):
         assert np.array_equal(outs[r], ref)
 
 
-@pytest.mark.parametrize("threads", [64, 256, 512])
+@pytest.mark.parametrize("threads", [32, 64, 256, 512])
 def test_parity_threads(comm, threads):
     comm(4, "single", 8192, channels=2, threads=threads)
     xs, outs = _run(4, "single", "bfloat16", 40000 + 3, 8192)
@@ -83,8 +88,10 @@ def test_parity_threads(comm, threads):
 
 def test_repeated_calls_advance_epochs(comm):
     comm(8, "double", 4096, channels=4)
-    for it in range(4):
-        count = [5000, 20000, 7, 12345][it]
+    for it in range(6):
+        if it == 3:
+            ccube.set_transport("push")   # params rebuilt, counters keep advancing
+        count = [5000, 20000, 7, 12345, 99, 40000][it]
         xs, outs = _run(8, "double", "float32", count, 4096, seed=100 + it)
         ref = oar.reference(xs, "double", 4096, "float32")[0]
         for r in range(8):
@@ -165,12 +172,13 @@ def _full_size(P, kind, dtype, workload, chunk_bytes, overlap=True):
 
 
 @pytest.mark.parametrize("kind", ["single", "double"])
-def test_full_size_resnet50_fp32(comm, kind):
+@pytest.mark.parametrize("transport", ["auto", "push"])
+def test_full_size_resnet50_fp32(comm, kind, transport):
     """configs[1]: ResNet-50 gradient set (25,557,032 fp32, K = 390) at P = 8 with the
     bench's launch configuration; sampled chunks bit-exact vs the oracle (first,
     last ragged, random), every rank identical, fp64 normwise error <= 1e-6."""
     P, chunk = 8, 256 << 10
-    comm(P, kind, chunk)
+    comm(P, kind, chunk, transport=transport)
     count, ends, ts = _full_size(P, kind, "float32", "resnet50", chunk)
     K = partition.num_chunks(count, chunk, 4)
     assert K == 390

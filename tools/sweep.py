@@ -26,6 +26,7 @@ def main():
     p.add_argument("--threads", default="512")
     p.add_argument("--chunks", default=str(256 << 10))
     p.add_argument("--iters", type=int, default=20)
+    p.add_argument("--transport", default="auto")
     p.add_argument("--bytes", type=int, default=0, help="override buffer bytes per rank")
     a = p.parse_args()
     tdt = {"float32": torch.float32, "bfloat16": torch.bfloat16, "int32": torch.int32}[a.dtype]
@@ -35,14 +36,15 @@ def main():
     bufs = [torch.randn(count, device="cuda").to(tdt) for _ in range(P)]
     flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
     s = torch.cuda.Stream()
-    for tree, ov, ch, th, cb in itertools.product(a.trees.split(","), a.overlap.split(","),
-                                                  a.channels.split(","), a.threads.split(","),
-                                                  a.chunks.split(",")):
+    for tree, ov, ch, th, cb, tp in itertools.product(a.trees.split(","), a.overlap.split(","),
+                                                      a.channels.split(","), a.threads.split(","),
+                                                      a.chunks.split(","), a.transport.split(",")):
         try:
             ccube.init_loopback(P, tree, int(cb))
             ccube.set_channels(int(ch))
             ccube.set_threads(int(th))
             ccube.set_overlap(bool(int(ov)))
+            ccube.set_transport(tp)
             ms = []
             for i in range(a.iters + 3):
                 with torch.cuda.stream(s):
@@ -58,7 +60,7 @@ def main():
             nbytes = count * es
             busbw = nbytes / (med / 1e3) / 1e9 * 2 * (P - 1) / P
             hbm = 2 * P * nbytes / (med / 1e3) / 1e9
-            print(json.dumps({"tree": tree, "overlap": int(ov), "channels": int(ch),
+            print(json.dumps({"tree": tree, "transport": tp, "overlap": int(ov), "channels": int(ch),
                               "threads": int(th), "chunk": int(cb), "ms": round(med, 4),
                               "busbw": round(busbw, 1), "hbm_algo_gbs": round(hbm, 1)}),
                   flush=True)
