@@ -155,7 +155,7 @@ struct Comm {
   int ntrees = 1;
   size_t chunk_bytes = CCUBE_DEFAULT_CHUNK_BYTES;
   Tree trees[kMaxTrees];
-  int channels = 8, threads = 512, overlap = 1;
+  int channels = 0, threads = 256, overlap = 1;  // channels 0 = auto
   uint64_t base[kMaxTrees] = {0, 0};
   bool have_call = false;
   uint64_t last_base[kMaxTrees] = {0, 0};
@@ -435,14 +435,31 @@ ccube_result_t get_tasks(int channels, int overlap, TaskTable **out) {
   return CCUBE_SUCCESS;
 }
 
-ccube_result_t check_chunk_channels(size_t chunk_bytes, int channels) {
-  if (chunk_bytes == 0 || chunk_bytes % (16ull * channels))
-    return fail(CCUBE_ERR_INVALID_ARG,
-                "chunk_bytes (%zu) must be a positive multiple of 16 * channels (%d)",
-                chunk_bytes, channels);
+ccube_result_t check_chunk(size_t chunk_bytes) {
+  if (chunk_bytes == 0 || chunk_bytes % 16)
+    return fail(CCUBE_ERR_INVALID_ARG, "chunk_bytes (%zu) must be a positive multiple of 16",
+                chunk_bytes);
   if (chunk_bytes > (1ull << 31))
     return fail(CCUBE_ERR_INVALID_ARG, "chunk_bytes (%zu) too large", chunk_bytes);
   return CCUBE_SUCCESS;
+}
+
+int count_tasks(int channels, int overlap) {
+  int n = 0;
+  for (int i = 0; i < g.nlocal; ++i) {
+    const int r = g.rank0 + i;
+    for (int t = 0; t < g.ntrees; ++t) {
+      const Tree &tr = g.trees[t];
+      const bool root = tr.parent[r] < 0;
+      if (!root && tr.nchild[r] == 0 && edge_is_pull(r, tr.parent[r])) {
+        n += 1;
+        continue;
+      }
+      n += channels;
+      if (tr.nchild[r] > 0 && (!root || !overlap)) n += channels;
+    }
+  }
+  return n;
 }
 
 ccube_result_t allreduce_impl(void *const *bufs, size_t count, ccube_dtype_t dtype,
@@ -466,31 +483,7 @@ ccube_result_t allreduce_impl(void *const *bufs, size_t count, ccube_dtype_t dty
 
   const uint64_t E = g.chunk_bytes / es;
   const uint64_t K = (count + E - 1) / E;
-  LaunchArgs a;
-  memset(&a, 0, sizeof a);
-  a.count = count;
-  a.elems_per_chunk = static_cast<uint32_t>(E);
-  a.slice_elems = static_cast<uint32_t>(E / g.channels);
-  a.ntrees = g.ntrees;
-  a.nchannels = g.channels;
-  if (g.ntrees == 1) {
-    a.K[0] = static_cast<uint32_t>(K);
-  } else {
-    a.K[0] = static_cast<uint32_t>((K + 1) / 2);
-    a.K[1] = static_cast<uint32_t>(K / 2);
-  }
   if (K > 0xffffffffull) return fail(CCUBE_ERR_INVALID_ARG, "too many chunks");
-  for (int t = 0; t < g.ntrees; ++t) a.base[t] = g.base[t];
-  a.overlap = g.overlap;
-  a.timeout_ns = g.timeout_ns;
-  a.err = g.err_dev;
-  a.trace = g.trace;
-  a.trace_kmax = static_cast<uint32_t>(g.trace_kmax);
-  a.params = R->d_params;
-
-  TaskTable *tt = nullptr;
-  CC_TRY(get_tasks(g.channels, g.overlap, &tt));
-  a.tasks = tt->d_tasks;
 
   // all CTAs spin on each other: they must be co-resident
   const int cta_threads = g.threads + 32;  // data warps + the control warp
@@ -504,10 +497,42 @@ ccube_result_t allreduce_impl(void *const *bufs, size_t count, ccube_dtype_t dty
     g.max_blocks[key] = b;
   }
   const int cap = g.max_blocks[key] * g.sm_count;
+  int J = g.channels;
+  if (J == 0) {  // auto: the most channels whose CTAs all fit at once
+    J = 1;
+    while (J < CCUBE_MAX_CHANNELS && count_tasks(J + 1, g.overlap) <= cap) ++J;
+  }
+  const uint64_t VE = 16 / es;
+  const uint64_t SL = ((E + J - 1) / J + VE - 1) / VE * VE;  // slice: 16 B multiple
+
+  LaunchArgs a;
+  memset(&a, 0, sizeof a);
+  a.count = count;
+  a.elems_per_chunk = static_cast<uint32_t>(E);
+  a.slice_elems = static_cast<uint32_t>(SL);
+  a.ntrees = g.ntrees;
+  a.nchannels = J;
+  if (g.ntrees == 1) {
+    a.K[0] = static_cast<uint32_t>(K);
+  } else {
+    a.K[0] = static_cast<uint32_t>((K + 1) / 2);
+    a.K[1] = static_cast<uint32_t>(K / 2);
+  }
+  for (int t = 0; t < g.ntrees; ++t) a.base[t] = g.base[t];
+  a.overlap = g.overlap;
+  a.timeout_ns = g.timeout_ns;
+  a.err = g.err_dev;
+  a.trace = g.trace;
+  a.trace_kmax = static_cast<uint32_t>(g.trace_kmax);
+  a.params = R->d_params;
+
+  TaskTable *tt = nullptr;
+  CC_TRY(get_tasks(J, g.overlap, &tt));
+  a.tasks = tt->d_tasks;
   if (tt->n > cap)
     return fail(CCUBE_ERR_UNSUPPORTED,
                 "%d CTAs (channels=%d) cannot be co-resident (capacity %d); lower channels",
-                tt->n, g.channels, cap);
+                tt->n, J, cap);
 
   const int rc = launch_tree_allreduce(a, dtype, g.sys_scope, tt->n, cta_threads, stream);
   if (rc != cudaSuccess)
@@ -515,7 +540,7 @@ ccube_result_t allreduce_impl(void *const *bufs, size_t count, ccube_dtype_t dty
                 cudaGetErrorString(static_cast<cudaError_t>(rc)));
   g.have_call = true;
   g.last_E = E;
-  g.last_channels = g.channels;
+  g.last_channels = J;
   for (int t = 0; t < g.ntrees; ++t) {
     g.last_base[t] = g.base[t];
     g.last_K[t] = a.K[t];
@@ -628,13 +653,13 @@ ccube_result_t ccube_init(const ccube_world_t *world, ccube_tree_kind_t tree_kin
   if (world->nlocal < P && !world->allgather)
     return fail(CCUBE_ERR_INVALID_ARG, "allgather callback required when nlocal < world_size");
   if (chunk_bytes == 0) chunk_bytes = CCUBE_DEFAULT_CHUNK_BYTES;
-  int channels = env_int("CCUBE_CHANNELS", 8);
-  if (channels < 1 || channels > CCUBE_MAX_CHANNELS)
+  int channels = env_int("CCUBE_CHANNELS", 0);
+  if (channels < 0 || channels > CCUBE_MAX_CHANNELS)
     return fail(CCUBE_ERR_INVALID_ARG, "CCUBE_CHANNELS %d out of range", channels);
-  CC_TRY(check_chunk_channels(chunk_bytes, channels));
-  int threads = env_int("CCUBE_THREADS", 512);
-  if (threads < 32 || threads > 512 || threads % 32)
-    return fail(CCUBE_ERR_INVALID_ARG, "CCUBE_THREADS %d out of range [32, 512]", threads);
+  CC_TRY(check_chunk(chunk_bytes));
+  int threads = env_int("CCUBE_THREADS", 256);
+  if (threads < 32 || threads > 256 || threads % 32)
+    return fail(CCUBE_ERR_INVALID_ARG, "CCUBE_THREADS %d out of range [32, 256]", threads);
   const int transport = env_int("CCUBE_TRANSPORT", CCUBE_TRANSPORT_AUTO);
   if (transport < CCUBE_TRANSPORT_AUTO || transport > CCUBE_TRANSPORT_PULL)
     return fail(CCUBE_ERR_INVALID_ARG, "CCUBE_TRANSPORT %d out of range", transport);
@@ -819,11 +844,10 @@ ccube_result_t ccube_set_overlap(int on) {
 ccube_result_t ccube_set_channels(int channels) {
   std::lock_guard<std::mutex> lk(g_mu);
   if (!g.init) return fail(CCUBE_ERR_NOT_INITIALIZED, "ccube_init has not been called");
-  if (channels == 0) channels = env_int("CCUBE_CHANNELS", 8);
-  if (channels < 1 || channels > CCUBE_MAX_CHANNELS)
-    return fail(CCUBE_ERR_INVALID_ARG, "channels %d out of range [1, %d]", channels,
+  if (channels < 0 || channels > CCUBE_MAX_CHANNELS)
+    return fail(CCUBE_ERR_INVALID_ARG, "channels %d out of range [0 (auto), %d]", channels,
                 CCUBE_MAX_CHANNELS);
-  CC_TRY(check_chunk_channels(g.chunk_bytes, channels));
+  
   g.channels = channels;
   return CCUBE_SUCCESS;
 }
@@ -831,8 +855,8 @@ ccube_result_t ccube_set_channels(int channels) {
 ccube_result_t ccube_set_threads(int threads) {
   std::lock_guard<std::mutex> lk(g_mu);
   if (!g.init) return fail(CCUBE_ERR_NOT_INITIALIZED, "ccube_init has not been called");
-  if (threads < 32 || threads > 512 || threads % 32)
-    return fail(CCUBE_ERR_INVALID_ARG, "threads %d out of range [32, 512] (multiple of 32)",
+  if (threads < 32 || threads > 256 || threads % 32)
+    return fail(CCUBE_ERR_INVALID_ARG, "threads %d out of range [32, 256] (multiple of 32)",
                 threads);
   g.threads = threads;
   return CCUBE_SUCCESS;

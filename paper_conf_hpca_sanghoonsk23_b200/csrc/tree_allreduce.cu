@@ -36,9 +36,8 @@
 namespace ccube {
 namespace {
 
-constexpr int kUnroll = 4;
-constexpr int kMaxThreads = 544;  // 16 data warps + the control warp
-constexpr int kMaxDataWarps = 16;
+constexpr int kMaxThreads = 288;  // up to 8 data warps + the control warp
+constexpr int kMaxDataWarps = 8;
 
 __device__ __forceinline__ uint64_t globaltimer() {
   uint64_t t;
@@ -233,91 +232,6 @@ struct Combine<kBFloat16> {
   }
 };
 
-// One data warp's share of elements [elo, ehi): vectors w*32+lane, stepping W*32,
-// U vectors per source in flight; the ragged scalar tail goes to warp 0.
-// Sources are local HBM or (PULL) peer buffers; destinations may be peer memory.
-template <int DT, int NIN, int NOUT>
-__device__ __forceinline__ void process_warp(const char *const *src, char *const *dst,
-                                             uint64_t elo, uint64_t ehi, int w, int W) {
-  constexpr int ES = DT == kBFloat16 ? 2 : 4;
-  constexpr int VE = 16 / ES;
-  if (ehi <= elo) return;
-  const uint64_t n = ehi - elo;
-  const uint64_t nv = n / VE;
-  const int lane = threadIdx.x & 31;
-  const uint4 *s[NIN];
-  uint4 *d[NOUT];
-#pragma unroll
-  for (int i = 0; i < NIN; ++i) s[i] = reinterpret_cast<const uint4 *>(src[i] + elo * ES);
-#pragma unroll
-  for (int i = 0; i < NOUT; ++i) d[i] = reinterpret_cast<uint4 *>(dst[i] + elo * ES);
-  const uint64_t step = static_cast<uint64_t>(W) * 32;
-  uint64_t i = static_cast<uint64_t>(w) * 32 + lane;
-  for (; i + (kUnroll - 1) * step < nv; i += kUnroll * step) {
-    uint4 v[kUnroll][NIN];
-#pragma unroll
-    for (int u = 0; u < kUnroll; ++u)
-#pragma unroll
-      for (int q = 0; q < NIN; ++q) v[u][q] = __ldcg(s[q] + i + u * step);
-#pragma unroll
-    for (int u = 0; u < kUnroll; ++u) {
-      const uint4 r = Combine<DT>::template vec<NIN>(v[u]);
-#pragma unroll
-      for (int q = 0; q < NOUT; ++q) d[q][i + u * step] = r;
-    }
-  }
-  for (; i < nv; i += step) {
-    uint4 v[NIN];
-#pragma unroll
-    for (int q = 0; q < NIN; ++q) v[q] = __ldcg(s[q] + i);
-    const uint4 r = Combine<DT>::template vec<NIN>(v);
-#pragma unroll
-    for (int q = 0; q < NOUT; ++q) d[q][i] = r;
-  }
-  if (w == 0) {
-    const char *ss[NIN];
-    char *dd[NOUT];
-#pragma unroll
-    for (int q = 0; q < NIN; ++q) ss[q] = src[q] + elo * ES;
-#pragma unroll
-    for (int q = 0; q < NOUT; ++q) dd[q] = dst[q] + elo * ES;
-    for (uint64_t e = nv * VE + lane; e < n; e += 32)
-      Combine<DT>::template scalar<NIN>(ss, dd, NOUT, e);
-  }
-}
-
-template <int DT, int NIN>
-__device__ __forceinline__ void process_nout(const char *const *src, char *const *dst, int nout,
-                                             uint64_t elo, uint64_t ehi, int w, int W) {
-  switch (nout) {
-    case 1: process_warp<DT, NIN, 1>(src, dst, elo, ehi, w, W); break;
-    case 2: process_warp<DT, NIN, 2>(src, dst, elo, ehi, w, W); break;
-    case 3: process_warp<DT, NIN, 3>(src, dst, elo, ehi, w, W); break;
-    default: break;
-  }
-}
-
-template <int DT>
-__device__ __forceinline__ void dispatch(const char *const *src, int nin, char *const *dst,
-                                         int nout, uint64_t elo, uint64_t ehi, int w, int W) {
-  switch (nin) {
-    case 1: process_nout<DT, 1>(src, dst, nout, elo, ehi, w, W); break;
-    case 2: process_nout<DT, 2>(src, dst, nout, elo, ehi, w, W); break;
-    case 3: process_nout<DT, 3>(src, dst, nout, elo, ehi, w, W); break;
-    default: break;
-  }
-}
-
-__device__ __forceinline__ void slice_range(const LaunchArgs &a, int t, int j, uint32_t k,
-                                            uint64_t *lo, uint64_t *hi) {
-  const uint64_t c = static_cast<uint64_t>(k) * a.ntrees + t;  // R4: chunk c on tree c mod T
-  const uint64_t cend = min((c + 1) * a.elems_per_chunk, a.count);
-  const uint64_t l = c * a.elems_per_chunk + static_cast<uint64_t>(j) * a.slice_elems;
-  const uint64_t h = min(l + a.slice_elems, cend);
-  *lo = l;
-  *hi = h > l ? h : l;
-}
-
 __device__ __forceinline__ void trace_landing(const LaunchArgs &a, int local, int t, uint32_t k0,
                                               uint32_t k1, int j) {
   if (a.trace == nullptr || local < 0) return;
@@ -438,14 +352,162 @@ __device__ void pulled_leaf(const LaunchArgs &a, const TreeParams &p, int t) {
   }
 }
 
-// ---- data warps ----------------------------------------------------------------
+// ---- data warps (TMA-staged) ------------------------------------------------------
+// A CTA's work for tree t, channel j is the sequence of its slices (slice j of every
+// tree-local chunk), cut into kSeg-byte segments; segment G belongs to data warp
+// G mod W.  Each warp runs its own kStages-deep ring: lane 0 issues one
+// cp.async.bulk (global -> shared, mbarrier complete_tx) per source as soon as the
+// segment's chunk is ready, then all lanes combine the staged sources (LDS.128),
+// and store the result with 128-bit STG into every destination (local or peer).
+// Loads stay in flight across chunk boundaries, so a warp never drains at a chunk.
+constexpr int kSeg = 2048;     // bytes per segment and source
+constexpr int kStages = 4;     // ring depth per data warp
+constexpr int kMaxIn = 1 + kMaxChildren;
+
+__device__ __forceinline__ uint32_t smem_u32(const void *p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+
+__device__ __forceinline__ void mbar_init(uint64_t *bar) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(bar)) : "memory");
+}
+
+__device__ __forceinline__ void mbar_expect_tx(uint64_t *bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)),
+               "r"(bytes)
+               : "memory");
+}
+
+__device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
+  uint32_t ok = 0;
+  while (!ok) {
+    asm volatile(
+        "{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2; "
+        "selp.u32 %0, 1, 0, p; }"
+        : "=r"(ok)
+        : "r"(smem_u32(bar)), "r"(parity)
+        : "memory");
+  }
+}
+
+__device__ __forceinline__ void bulk_load(void *smem_dst, const void *gmem_src, uint32_t bytes,
+                                          uint64_t *bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+          smem_u32(smem_dst)),
+      "l"(gmem_src), "r"(bytes), "r"(smem_u32(bar))
+      : "memory");
+}
+
+// Geometry of one (tree, channel) stream of segments, identical in every warp.
+struct SegMap {
+  uint64_t chunk_stride;  // bytes between consecutive tree-local chunks (T * E_b)
+  uint64_t first;         // byte offset of slice j of tree-local chunk 0
+  uint32_t nseg;          // segments per full slice
+  uint32_t kfull;         // tree-local chunks with a full-length slice
+  uint32_t sl_full;       // bytes of a full slice for this channel
+  uint32_t nseg_last;     // segments of the last (short) chunk, incl. a ragged one
+  uint32_t last_len;      // bytes of the last chunk's slice (may end off a 16 B boundary)
+  uint32_t total;         // kfull * nseg + nseg_last
+};
+
+template <int ES>
+__device__ __forceinline__ SegMap seg_map(const LaunchArgs &a, int t, int j) {
+  SegMap m;
+  const uint64_t Eb = static_cast<uint64_t>(a.elems_per_chunk) * ES;
+  const uint64_t SLb = static_cast<uint64_t>(a.slice_elems) * ES;
+  const uint64_t jo = static_cast<uint64_t>(j) * SLb;
+  m.chunk_stride = Eb * a.ntrees;
+  m.first = static_cast<uint64_t>(t) * Eb + jo;
+  m.sl_full = static_cast<uint32_t>(jo < Eb ? min(SLb, Eb - jo) : 0);
+  m.nseg = (m.sl_full + kSeg - 1) / kSeg;
+  const uint32_t K = a.K[t];
+  const uint64_t nbytes = a.count * ES;
+  const uint64_t Ktot = (a.count + a.elems_per_chunk - 1) / a.elems_per_chunk;
+  const uint64_t C = Ktot - 1;  // last global chunk
+  m.kfull = K;
+  m.last_len = 0;
+  m.nseg_last = 0;
+  if (K > 0 && (C % a.ntrees) == static_cast<uint64_t>(t) && nbytes < (C + 1) * Eb) {
+    m.kfull = K - 1;  // this tree carries the short last chunk
+    const uint64_t s0 = C * Eb + jo;
+    m.last_len = static_cast<uint32_t>(s0 < nbytes ? min(SLb, nbytes - s0) : 0);
+    const uint32_t aligned = m.last_len & ~15u;
+    m.nseg_last = (aligned + kSeg - 1) / kSeg + ((m.last_len & 15u) ? 1 : 0);
+  }
+  m.total = m.nseg ? m.kfull * m.nseg + m.nseg_last : m.nseg_last;
+  return m;
+}
+
+__device__ __forceinline__ uint32_t seg_chunk(const SegMap &m, uint32_t G) {
+  if (m.nseg == 0) return m.kfull;
+  const uint32_t k = G / m.nseg;
+  return k < m.kfull ? k : m.kfull;
+}
+
+// byte offset within the buffer and length of segment G; len < 16 marks the
+// ragged sub-vector tail at the very end of the buffer (scalar path, no TMA)
+__device__ __forceinline__ void seg_range(const SegMap &m, uint32_t G, uint64_t *off,
+                                          uint32_t *len) {
+  const uint32_t k = seg_chunk(m, G);
+  const uint32_t s = G - k * m.nseg;
+  const uint64_t base = m.first + static_cast<uint64_t>(k) * m.chunk_stride;
+  if (k < m.kfull) {
+    *off = base + static_cast<uint64_t>(s) * kSeg;
+    *len = min(static_cast<uint32_t>(kSeg), m.sl_full - s * kSeg);
+    return;
+  }
+  const uint32_t aligned = m.last_len & ~15u;
+  const uint32_t full_segs = (aligned + kSeg - 1) / kSeg;
+  if (s < full_segs) {
+    *off = base + static_cast<uint64_t>(s) * kSeg;
+    *len = min(static_cast<uint32_t>(kSeg), aligned - s * kSeg);
+  } else {
+    *off = base + aligned;
+    *len = m.last_len - aligned;  // 1..15 bytes
+  }
+}
+
+template <int DT, int NIN>
+__device__ __forceinline__ void combine_stage(const char *stage, uint32_t len, char *const *dst,
+                                              int nout, uint64_t off) {
+  const int lane = threadIdx.x & 31;
+  for (uint32_t v = lane; v < len / 16; v += 32) {
+    uint4 x[NIN];
+#pragma unroll
+    for (int q = 0; q < NIN; ++q)
+      x[q] = *reinterpret_cast<const uint4 *>(stage + q * kSeg + v * 16);
+    const uint4 r = Combine<DT>::template vec<NIN>(x);
+    for (int d = 0; d < nout; ++d) *reinterpret_cast<uint4 *>(dst[d] + off + v * 16) = r;
+  }
+}
+
+template <int DT>
+__device__ __forceinline__ void combine_scalar(const char *const *src, int nin, char *const *dst,
+                                               int nout, uint64_t off, uint32_t len) {
+  constexpr int ES = DT == kBFloat16 ? 2 : 4;
+  const int lane = threadIdx.x & 31;
+  const char *ss[kMaxIn];
+  char *dd[kMaxIn];
+  for (int q = 0; q < nin; ++q) ss[q] = src[q] + off;
+  for (int q = 0; q < nout; ++q) dd[q] = dst[q] + off;
+  for (uint32_t e = lane; e < len / ES; e += 32) {
+    switch (nin) {
+      case 1: Combine<DT>::template scalar<1>(ss, dd, nout, e); break;
+      case 2: Combine<DT>::template scalar<2>(ss, dd, nout, e); break;
+      default: Combine<DT>::template scalar<3>(ss, dd, nout, e); break;
+    }
+  }
+}
+
 template <int DT>
 __device__ void data_warp(const LaunchArgs &a, const TreeParams &p, int role, int t, int j,
-                          int w, int W, Shared &sh) {
+                          int w, int W, Shared &sh, char *stage_base, uint64_t *bars) {
+  constexpr int ES = DT == kBFloat16 ? 2 : 4;
   const int lane = threadIdx.x & 31;
   const uint32_t K = a.K[t];
-  const char *src[3];
-  char *dst[3];
+  const char *src[kMaxIn];
+  char *dst[kMaxIn];
   int nin, nout;
   if (role == kRoleUp) {
     nin = 1 + p.nchild;
@@ -462,30 +524,84 @@ __device__ void data_warp(const LaunchArgs &a, const TreeParams &p, int role, in
     for (int s = 0; s < p.nchild; ++s) dst[s] = p.child_buf[s];
     nout = p.nchild;
   }
-  uint64_t ready = 0;
-  for (uint32_t k = 0; k < K; ++k) {
-    if (ready <= k) {
-      uint64_t r = 0;
-      if (lane == 0) {
-        do {
-          r = ld_acquire_cta(&sh.ready);
-        } while (r <= k && !*reinterpret_cast<volatile int *>(&sh.abort));
-      }
-      r = __shfl_sync(0xffffffffu, r, 0);
-      if (r <= k) return;  // aborted
-      ready = r;
-    }
-    uint64_t lo, hi;
-    slice_range(a, t, j, k, &lo, &hi);
-    dispatch<DT>(src, nin, dst, nout, lo, hi, w, W);
-    __syncwarp();
-    if (lane == 0) st_release_cta(&sh.done[w], k + 1);
+  const SegMap m = seg_map<ES>(a, t, j);
+  const uint32_t mine = m.total > static_cast<uint32_t>(w)
+                            ? (m.total - w + W - 1) / W : 0;  // segments w, w+W, ...
+  char *my_stages = stage_base + static_cast<size_t>(w) * kStages * kMaxIn * kSeg;
+  uint64_t *my_bars = bars + w * kStages;
+  if (lane == 0) {
+    for (int s = 0; s < kStages; ++s) mbar_init(&my_bars[s]);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
+  __syncwarp();
+
+  uint32_t issued = 0, consumed = 0, done_reported = 0;
+  uint64_t ready = 0;
+  while (consumed < mine) {
+    // issue every segment whose chunk is ready, up to kStages ahead
+    while (issued < mine && issued - consumed < kStages) {
+      const uint32_t G = w + issued * W;
+      const uint32_t k = seg_chunk(m, G);
+      if (k >= ready) {
+        if (issued > consumed) break;  // work is staged: consume it first
+        uint64_t r = 0;
+        if (lane == 0) {
+          do {
+            r = ld_acquire_cta(&sh.ready);
+          } while (r <= k && !*reinterpret_cast<volatile int *>(&sh.abort));
+          // order the generic-proxy acquire before the async-proxy (TMA) reads
+          asm volatile("fence.proxy.async.global;" ::: "memory");
+        }
+        r = __shfl_sync(0xffffffffu, r, 0);
+        if (r <= k) return;  // aborted
+        ready = r;
+      }
+      uint64_t off;
+      uint32_t len;
+      seg_range(m, G, &off, &len);
+      if (lane == 0 && len >= 16) {
+        const int st = issued % kStages;
+        char *buf = my_stages + static_cast<size_t>(st) * kMaxIn * kSeg;
+        mbar_expect_tx(&my_bars[st], len * nin);
+        for (int q = 0; q < nin; ++q) bulk_load(buf + q * kSeg, src[q] + off, len, &my_bars[st]);
+      }
+      ++issued;
+    }
+    // consume the oldest staged segment
+    {
+      const uint32_t G = w + consumed * W;
+      uint64_t off;
+      uint32_t len;
+      seg_range(m, G, &off, &len);
+      const int st = consumed % kStages;
+      if (len >= 16) {
+        mbar_wait(&my_bars[st], (consumed / kStages) & 1);
+        const char *buf = my_stages + static_cast<size_t>(st) * kMaxIn * kSeg;
+        switch (nin) {
+          case 1: combine_stage<DT, 1>(buf, len, dst, nout, off); break;
+          case 2: combine_stage<DT, 2>(buf, len, dst, nout, off); break;
+          default: combine_stage<DT, 3>(buf, len, dst, nout, off); break;
+        }
+      } else {
+        combine_scalar<DT>(src, nin, dst, nout, off, len);
+      }
+      __syncwarp();  // every lane is done with the stage and has issued its stores
+      ++consumed;
+      const uint32_t d = consumed < mine ? seg_chunk(m, w + consumed * W) : K;
+      if (d > done_reported) {
+        if (lane == 0) st_release_cta(&sh.done[w], d);
+        done_reported = d;
+      }
+    }
+  }
+  if (done_reported < K && lane == 0) st_release_cta(&sh.done[w], K);
 }
 
 template <int DT, bool SYS>
 __global__ void __launch_bounds__(kMaxThreads) tree_allreduce_kernel(const LaunchArgs a) {
   __shared__ Shared sh;
+  __shared__ uint64_t bars[kMaxDataWarps * kStages];
+  extern __shared__ __align__(128) char stages[];
   const Task task = a.tasks[blockIdx.x];
   const TreeParams &p = a.params[task.local_rank * a.ntrees + task.tree];
   const int warp = threadIdx.x >> 5;
@@ -503,7 +619,7 @@ __global__ void __launch_bounds__(kMaxThreads) tree_allreduce_kernel(const Launc
   if (warp == 0)
     control_warp<SYS>(a, p, task.role, task.tree, task.channel, W, sh);
   else
-    data_warp<DT>(a, p, task.role, task.tree, task.channel, warp - 1, W, sh);
+    data_warp<DT>(a, p, task.role, task.tree, task.channel, warp - 1, W, sh, stages, bars);
 }
 
 struct GateArgs {
@@ -530,9 +646,18 @@ __global__ void gate_kernel(const GateArgs g) {
   }
 }
 
+size_t stage_bytes(int threads) {
+  return static_cast<size_t>(threads / 32 - 1) * kStages * kMaxIn * kSeg;
+}
+
 template <int DT, bool SYS>
 int launch_t(const LaunchArgs &a, int grid, int threads, cudaStream_t s) {
-  tree_allreduce_kernel<DT, SYS><<<grid, threads, 0, s>>>(a);
+  const size_t smem = stage_bytes(threads);
+  cudaError_t e = cudaFuncSetAttribute(tree_allreduce_kernel<DT, SYS>,
+                                       cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       static_cast<int>(smem));
+  if (e != cudaSuccess) return static_cast<int>(e);
+  tree_allreduce_kernel<DT, SYS><<<grid, threads, smem, s>>>(a);
   return static_cast<int>(cudaGetLastError());
 }
 
@@ -597,7 +722,11 @@ int query_max_blocks_per_sm(int dtype, bool sys_scope, int threads, int *blocks)
       fn = sys_scope ? kernel_ptr<kBFloat16, true>() : kernel_ptr<kBFloat16, false>();
       break;
   }
-  return static_cast<int>(cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks, fn, threads, 0));
+  const size_t smem = stage_bytes(threads);
+  cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       static_cast<int>(smem));
+  if (e != cudaSuccess) return static_cast<int>(e);
+  return static_cast<int>(cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks, fn, threads, smem));
 }
 
 }  // namespace ccube

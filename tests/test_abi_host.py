@@ -57,7 +57,7 @@ def test_calls_before_init_fail_cleanly():
     (dict(world_size=0), ccube.ERR_INVALID_ARG),
     (dict(world_size=4, nlocal=3), ccube.ERR_INVALID_ARG),
     (dict(world_size=4, chunk_bytes=1000), ccube.ERR_INVALID_ARG),
-    (dict(world_size=4, chunk_bytes=16 * 7), ccube.ERR_INVALID_ARG),   # not a multiple of 16*8
+    (dict(world_size=4, chunk_bytes=16 * 7 + 8), ccube.ERR_INVALID_ARG),   # not a multiple of 16
     (dict(world_size=4, rank=1), ccube.ERR_INVALID_ARG),
 ])
 def test_init_validation(kwargs, code):
