@@ -95,7 +95,7 @@ struct LaunchArgs {
   int *err;                   // mapped host word; nonzero = abort
   uint64_t *trace;            // optional landing trace
   uint32_t trace_kmax;
-  uint32_t pad1;
+  uint32_t seg_bytes;         // TMA segment bytes per source (stage size)
 };
 
 // Kernel launcher (tree_allreduce.cu).  Returns a cudaError_t as int.
@@ -104,6 +104,7 @@ int launch_tree_allreduce(const LaunchArgs &args, int dtype, bool sys_scope, int
 constexpr int kMaxGateCounters = 128;
 int launch_gate(const uint64_t *const *counters, const uint64_t *targets, int n, int *err,
                 uint64_t timeout_ns, bool sys_scope, void *stream);
-int query_max_blocks_per_sm(int dtype, bool sys_scope, int threads, int *blocks);
+int query_max_blocks_per_sm(int dtype, bool sys_scope, int threads, uint32_t seg_bytes,
+                            int *blocks);
 
 }  // namespace ccube

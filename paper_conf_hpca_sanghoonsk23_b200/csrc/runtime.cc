@@ -170,6 +170,7 @@ struct Comm {
   std::vector<std::unique_ptr<Registration>> regs;
   std::map<std::pair<int, int>, TaskTable> tasks;  // (channels, overlap)
   int transport = CCUBE_TRANSPORT_AUTO;
+  uint32_t seg_bytes = 16384;  // TMA stage bytes per source
   bool sys_scope = false;
   uint64_t timeout_ns = 10000ull * 1000000ull;
   int sm_count = 0;
@@ -487,10 +488,10 @@ ccube_result_t allreduce_impl(void *const *bufs, size_t count, ccube_dtype_t dty
 
   // all CTAs spin on each other: they must be co-resident
   const int cta_threads = g.threads + 32;  // data warps + the control warp
-  auto key = std::make_pair((int)dtype, cta_threads);
+  auto key = std::make_pair((int)dtype, cta_threads * 1024 + (int)(g.seg_bytes >> 4));
   if (!g.max_blocks.count(key)) {
     int b = 0;
-    const int rc = query_max_blocks_per_sm(dtype, g.sys_scope, cta_threads, &b);
+    const int rc = query_max_blocks_per_sm(dtype, g.sys_scope, cta_threads, g.seg_bytes, &b);
     if (rc != cudaSuccess)
       return fail(CCUBE_ERR_CUDA, "occupancy query failed: %s",
                   cudaGetErrorString(static_cast<cudaError_t>(rc)));
@@ -524,6 +525,7 @@ ccube_result_t allreduce_impl(void *const *bufs, size_t count, ccube_dtype_t dty
   a.err = g.err_dev;
   a.trace = g.trace;
   a.trace_kmax = static_cast<uint32_t>(g.trace_kmax);
+  a.seg_bytes = g.seg_bytes;
   a.params = R->d_params;
 
   TaskTable *tt = nullptr;
@@ -658,8 +660,8 @@ ccube_result_t ccube_init(const ccube_world_t *world, ccube_tree_kind_t tree_kin
     return fail(CCUBE_ERR_INVALID_ARG, "CCUBE_CHANNELS %d out of range", channels);
   CC_TRY(check_chunk(chunk_bytes));
   int threads = env_int("CCUBE_THREADS", 256);
-  if (threads < 32 || threads > 256 || threads % 32)
-    return fail(CCUBE_ERR_INVALID_ARG, "CCUBE_THREADS %d out of range [32, 256]", threads);
+  if (threads < 32 || threads > 512 || threads % 32)
+    return fail(CCUBE_ERR_INVALID_ARG, "CCUBE_THREADS %d out of range [32, 512]", threads);
   const int transport = env_int("CCUBE_TRANSPORT", CCUBE_TRANSPORT_AUTO);
   if (transport < CCUBE_TRANSPORT_AUTO || transport > CCUBE_TRANSPORT_PULL)
     return fail(CCUBE_ERR_INVALID_ARG, "CCUBE_TRANSPORT %d out of range", transport);
@@ -678,6 +680,11 @@ ccube_result_t ccube_init(const ccube_world_t *world, ccube_tree_kind_t tree_kin
   g.channels = channels;
   g.threads = threads;
   g.transport = transport;
+  g.seg_bytes = static_cast<uint32_t>(env_int("CCUBE_SEG_BYTES", 16384));
+  if (g.seg_bytes < 1024 || g.seg_bytes > 16384 || g.seg_bytes % 1024) {
+    g = Comm();
+    return fail(CCUBE_ERR_INVALID_ARG, "CCUBE_SEG_BYTES must be a multiple of 1024 in [1024, 16384]");
+  }
   g.overlap = 1;
   g.sys_scope = g.nproc > 1;
   g.timeout_ns = static_cast<uint64_t>(env_int("CCUBE_WATCHDOG_MS", 10000)) * 1000000ull;
@@ -855,8 +862,8 @@ ccube_result_t ccube_set_channels(int channels) {
 ccube_result_t ccube_set_threads(int threads) {
   std::lock_guard<std::mutex> lk(g_mu);
   if (!g.init) return fail(CCUBE_ERR_NOT_INITIALIZED, "ccube_init has not been called");
-  if (threads < 32 || threads > 256 || threads % 32)
-    return fail(CCUBE_ERR_INVALID_ARG, "threads %d out of range [32, 256] (multiple of 32)",
+  if (threads < 32 || threads > 512 || threads % 32)
+    return fail(CCUBE_ERR_INVALID_ARG, "threads %d out of range [32, 512] (multiple of 32)",
                 threads);
   g.threads = threads;
   return CCUBE_SUCCESS;

@@ -36,8 +36,8 @@
 namespace ccube {
 namespace {
 
-constexpr int kMaxThreads = 288;  // up to 8 data warps + the control warp
-constexpr int kMaxDataWarps = 8;
+constexpr int kMaxThreads = 544;  // up to 16 data warps + the control warp
+constexpr int kMaxDataWarps = 16;
 
 __device__ __forceinline__ uint64_t globaltimer() {
   uint64_t t;
@@ -71,21 +71,6 @@ __device__ __forceinline__ void st_relaxed(uint64_t *p, uint64_t v) {
     asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
 
-// CTA-scope release/acquire on shared memory (control <-> data warps)
-__device__ __forceinline__ void st_release_cta(uint64_t *p, uint64_t v) {
-  asm volatile("st.release.cta.shared.u64 [%0], %1;" ::"r"((uint32_t)__cvta_generic_to_shared(p)),
-               "l"(v)
-               : "memory");
-}
-__device__ __forceinline__ uint64_t ld_acquire_cta(const uint64_t *p) {
-  uint64_t v;
-  asm volatile("ld.acquire.cta.shared.u64 %0, [%1];"
-               : "=l"(v)
-               : "r"((uint32_t)__cvta_generic_to_shared(p))
-               : "memory");
-  return v;
-}
-
 __device__ __forceinline__ uint64_t warp_min(uint64_t v) {
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) {
@@ -94,12 +79,6 @@ __device__ __forceinline__ uint64_t warp_min(uint64_t v) {
   }
   return v;
 }
-
-struct Shared {
-  uint64_t ready;                 // chunks whose inputs are available (control -> data)
-  uint64_t done[kMaxDataWarps];   // chunks finished by data warp w (data -> control)
-  int abort;
-};
 
 // Watchdog bookkeeping for the control warp.
 struct Watch {
@@ -243,7 +222,176 @@ __device__ __forceinline__ void trace_landing(const LaunchArgs &a, int local, in
   }
 }
 
-// ---- control warp --------------------------------------------------------------
+// ---- TMA staging primitives ----------------------------------------------------------
+constexpr int kStages = 4;                 // ring depth (per CTA)
+constexpr int kMaxIn = 1 + kMaxChildren;   // sources of a combine
+
+__device__ __forceinline__ uint32_t smem_u32(const void *p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+
+__device__ __forceinline__ void mbar_init(uint64_t *bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count)
+               : "memory");
+}
+
+__device__ __forceinline__ void mbar_expect_tx(uint64_t *bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)),
+               "r"(bytes)
+               : "memory");
+}
+
+__device__ __forceinline__ void mbar_arrive(uint64_t *bar) {  // .release.cta
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+
+__device__ __forceinline__ bool mbar_test(uint64_t *bar, uint32_t parity) {  // .acquire.cta
+  uint32_t ok;
+  asm volatile(
+      "{ .reg .pred p; mbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2; "
+      "selp.u32 %0, 1, 0, p; }"
+      : "=r"(ok)
+      : "r"(smem_u32(bar)), "r"(parity)
+      : "memory");
+  return ok != 0;
+}
+
+// blocking wait that gives up when the producer aborted
+__device__ __forceinline__ bool mbar_wait(uint64_t *bar, uint32_t parity, const int *abort) {
+  uint32_t spins = 0;
+  while (true) {
+    uint32_t ok;
+    asm volatile(
+        "{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2; "
+        "selp.u32 %0, 1, 0, p; }"
+        : "=r"(ok)
+        : "r"(smem_u32(bar)), "r"(parity)
+        : "memory");
+    if (ok) return true;
+    if ((++spins & 15) == 0 && *reinterpret_cast<const volatile int *>(abort)) return false;
+  }
+}
+
+__device__ __forceinline__ void bulk_load(void *smem_dst, const void *gmem_src, uint32_t bytes,
+                                          uint64_t *bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+          smem_u32(smem_dst)),
+      "l"(gmem_src), "r"(bytes), "r"(smem_u32(bar))
+      : "memory");
+}
+
+// ---- segment geometry --------------------------------------------------------------
+// A CTA's work for (tree t, channel j) is slice j of every tree-local chunk, cut
+// into segments of at most a.seg_bytes per source, processed in order G = 0, 1, ...
+struct SegMap {
+  uint64_t chunk_stride;  // bytes between consecutive tree-local chunks (T * E_b)
+  uint64_t first;         // byte offset of slice j of tree-local chunk 0
+  uint32_t seg;           // segment bytes
+  uint32_t nseg;          // segments per full slice
+  uint32_t kfull;         // tree-local chunks with a full-length slice
+  uint32_t sl_full;       // bytes of a full slice of this channel
+  uint32_t nseg_last;     // segments of the short last chunk, incl. a ragged one
+  uint32_t last_len;      // bytes of the last chunk's slice (may end off a 16 B boundary)
+  uint32_t total;         // kfull * nseg + nseg_last
+};
+
+template <int ES>
+__device__ __forceinline__ SegMap seg_map(const LaunchArgs &a, int t, int j) {
+  SegMap m;
+  const uint64_t Eb = static_cast<uint64_t>(a.elems_per_chunk) * ES;
+  const uint64_t SLb = static_cast<uint64_t>(a.slice_elems) * ES;
+  const uint64_t jo = static_cast<uint64_t>(j) * SLb;
+  m.seg = a.seg_bytes;
+  m.chunk_stride = Eb * a.ntrees;
+  m.first = static_cast<uint64_t>(t) * Eb + jo;
+  m.sl_full = static_cast<uint32_t>(jo < Eb ? min(SLb, Eb - jo) : 0);
+  m.nseg = (m.sl_full + m.seg - 1) / m.seg;
+  const uint32_t K = a.K[t];
+  const uint64_t nbytes = a.count * ES;
+  const uint64_t Ktot = (a.count + a.elems_per_chunk - 1) / a.elems_per_chunk;
+  const uint64_t C = Ktot - 1;  // last global chunk
+  m.kfull = K;
+  m.last_len = 0;
+  m.nseg_last = 0;
+  if (K > 0 && (C % a.ntrees) == static_cast<uint64_t>(t) && nbytes < (C + 1) * Eb) {
+    m.kfull = K - 1;  // this tree carries the short last chunk
+    const uint64_t s0 = C * Eb + jo;
+    m.last_len = static_cast<uint32_t>(s0 < nbytes ? min(SLb, nbytes - s0) : 0);
+    const uint32_t aligned = m.last_len & ~15u;
+    m.nseg_last = (aligned + m.seg - 1) / m.seg + ((m.last_len & 15u) ? 1 : 0);
+  }
+  m.total = m.nseg ? m.kfull * m.nseg + m.nseg_last : m.nseg_last;
+  return m;
+}
+
+__device__ __forceinline__ uint32_t seg_chunk(const SegMap &m, uint32_t G) {
+  if (m.nseg == 0) return m.kfull;
+  const uint32_t k = G / m.nseg;
+  return k < m.kfull ? k : m.kfull;
+}
+
+// byte offset in the buffer and length of segment G; len < 16 marks the ragged
+// sub-vector tail at the very end of the buffer (scalar path, no TMA)
+__device__ __forceinline__ void seg_range(const SegMap &m, uint32_t G, uint64_t *off,
+                                          uint32_t *len) {
+  const uint32_t k = seg_chunk(m, G);
+  const uint32_t s = G - k * m.nseg;
+  const uint64_t base = m.first + static_cast<uint64_t>(k) * m.chunk_stride;
+  if (k < m.kfull) {
+    *off = base + static_cast<uint64_t>(s) * m.seg;
+    *len = min(m.seg, m.sl_full - s * m.seg);
+    return;
+  }
+  const uint32_t aligned = m.last_len & ~15u;
+  const uint32_t full_segs = (aligned + m.seg - 1) / m.seg;
+  if (s < full_segs) {
+    *off = base + static_cast<uint64_t>(s) * m.seg;
+    *len = min(m.seg, aligned - s * m.seg);
+  } else {
+    *off = base + aligned;
+    *len = m.last_len - aligned;  // 1..15 bytes
+  }
+}
+
+// Sources and destinations of a task (a4/a5/a6).
+struct Endpoints {
+  const char *src[kMaxIn];
+  char *dst[kMaxIn];
+  int nin, nout;
+};
+
+__device__ __forceinline__ Endpoints endpoints(const LaunchArgs &a, const TreeParams &p, int role) {
+  Endpoints e;
+  if (role == kRoleUp) {
+    e.nin = 1 + p.nchild;
+    for (int q = 0; q < e.nin; ++q) e.src[q] = p.up_src[q];
+    e.dst[0] = p.up_dst;
+    e.nout = 1;
+    if (p.is_root && a.overlap) {  // C1 turnaround: final straight into the children
+      for (int s = 0; s < p.nchild; ++s) e.dst[1 + s] = p.child_buf[s];
+      e.nout += p.nchild;
+    }
+  } else {
+    e.nin = 1;
+    e.src[0] = p.buf;
+    for (int s = 0; s < p.nchild; ++s) e.dst[s] = p.child_buf[s];
+    e.nout = p.nchild;
+  }
+  return e;
+}
+
+struct Shared {
+  uint64_t full[kStages];   // producer -> consumers: stage loaded (TMA complete_tx)
+  uint64_t empty[kStages];  // consumers -> producer: stage consumed, stores issued
+  int abort;
+};
+
+__device__ __forceinline__ char *stage_ptr(char *stages, uint32_t seg, int st, int q) {
+  return stages + (static_cast<size_t>(st) * kMaxIn + q) * seg;
+}
+
+// ---- control / producer warp -------------------------------------------------------
 // Releases chunks [pub, d) downstream: one fence, then one store per counter.
 template <bool SYS>
 __device__ __forceinline__ void publish(const LaunchArgs &a, const TreeParams &p, int role, int t,
@@ -266,13 +414,15 @@ __device__ __forceinline__ void publish(const LaunchArgs &a, const TreeParams &p
   }
 }
 
-template <bool SYS>
+template <int ES, bool SYS>
 __device__ void control_warp(const LaunchArgs &a, const TreeParams &p, int role, int t, int j,
-                             int W, Shared &sh) {
+                             Shared &sh, char *stages) {
   const int lane = threadIdx.x & 31;
   const uint32_t K = a.K[t];
   const uint64_t base = a.base[t];
   const int stride = j * kFlagStrideU64;
+  const Endpoints e = endpoints(a, p, role);
+  const SegMap m = seg_map<ES>(a, t, j);
   // upstream counters: UP waits on each child's head, DOWN on my own semaphore
   const uint64_t *up = nullptr;
   if (role == kRoleUp) {
@@ -282,30 +432,64 @@ __device__ void control_warp(const LaunchArgs &a, const TreeParams &p, int role,
   }
   const bool hold_all = role == kRoleDown && p.is_root;  // B-mode root (Obs #1)
   uint64_t ready = (role == kRoleUp && p.nchild == 0) ? K : 0;  // a leaf's input is ready
-  if (lane == 0) st_release_cta(&sh.ready, ready);
-  uint32_t pub = 0;
+  bool fresh = true;  // ready advanced since the last proxy fence
+  uint32_t issued = 0, retired = 0, pub = 0;
   Watch wd;
   watch_reset(wd);
   while (pub < K) {
     bool moved = false;
-    if (ready < K) {
+    // (1) readiness: poll upstream (one lane per child, .gpu/.sys acquire)
+    const uint32_t need = issued < m.total ? seg_chunk(m, issued) : K;
+    if (ready < K && need >= ready) {
       uint64_t v = up ? ld_acquire<SYS>(up) : ~0ull;
       v = warp_min(v);
       uint64_t r = v > base ? v - base : 0;
       if (r > K) r = K;
       if (hold_all && r < K) r = 0;
       if (r > ready) {
+        __syncwarp();  // every lane's acquire is ordered before lane 0's TMA issue
         ready = r;
-        if (lane == 0) st_release_cta(&sh.ready, ready);
+        fresh = true;
         moved = true;
       }
     }
-    uint64_t d = lane < W ? ld_acquire_cta(&sh.done[lane]) : ~0ull;
-    d = warp_min(d);
+    // (2) issue TMA loads for ready segments into free stages
+    if (lane == 0) {
+      while (issued < m.total && issued - retired < kStages) {
+        const uint32_t k = seg_chunk(m, issued);
+        if (k >= ready) break;
+        if (fresh) {  // generic-proxy acquire -> async-proxy (TMA) reads
+          asm volatile("fence.proxy.async.global;" ::: "memory");
+          fresh = false;
+        }
+        uint64_t off;
+        uint32_t len;
+        seg_range(m, issued, &off, &len);
+        const int st = issued % kStages;
+        if (len >= 16) {
+          mbar_expect_tx(&sh.full[st], len * e.nin);
+          for (int q = 0; q < e.nin; ++q)
+            bulk_load(stage_ptr(stages, m.seg, st, q), e.src[q] + off, len, &sh.full[st]);
+        } else {
+          mbar_arrive(&sh.full[st]);  // ragged tail: consumers read it from global
+        }
+        ++issued;
+        moved = true;
+      }
+      // (3) retire stages the consumers have finished (non-blocking)
+      while (retired < issued && mbar_test(&sh.empty[retired % kStages], (retired / kStages) & 1)) {
+        ++retired;
+        moved = true;
+      }
+    }
+    issued = __shfl_sync(0xffffffffu, issued, 0);
+    retired = __shfl_sync(0xffffffffu, retired, 0);
+    fresh = __shfl_sync(0xffffffffu, fresh, 0);
+    // (4) a chunk is done once every segment of it is retired
+    const uint32_t d = retired < m.total ? seg_chunk(m, retired) : K;
     if (d > pub) {
-      __syncwarp();
-      if (lane == 0) publish<SYS>(a, p, role, t, j, pub, static_cast<uint32_t>(d), base);
-      pub = static_cast<uint32_t>(d);
+      if (lane == 0) publish<SYS>(a, p, role, t, j, pub, d, base);
+      pub = d;
       moved = true;
     }
     if (moved) {
@@ -352,131 +536,18 @@ __device__ void pulled_leaf(const LaunchArgs &a, const TreeParams &p, int t) {
   }
 }
 
-// ---- data warps (TMA-staged) ------------------------------------------------------
-// A CTA's work for tree t, channel j is the sequence of its slices (slice j of every
-// tree-local chunk), cut into kSeg-byte segments; segment G belongs to data warp
-// G mod W.  Each warp runs its own kStages-deep ring: lane 0 issues one
-// cp.async.bulk (global -> shared, mbarrier complete_tx) per source as soon as the
-// segment's chunk is ready, then all lanes combine the staged sources (LDS.128),
-// and store the result with 128-bit STG into every destination (local or peer).
-// Loads stay in flight across chunk boundaries, so a warp never drains at a chunk.
-constexpr int kSeg = 2048;     // bytes per segment and source
-constexpr int kStages = 4;     // ring depth per data warp
-constexpr int kMaxIn = 1 + kMaxChildren;
-
-__device__ __forceinline__ uint32_t smem_u32(const void *p) {
-  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
-}
-
-__device__ __forceinline__ void mbar_init(uint64_t *bar) {
-  asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(bar)) : "memory");
-}
-
-__device__ __forceinline__ void mbar_expect_tx(uint64_t *bar, uint32_t bytes) {
-  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)),
-               "r"(bytes)
-               : "memory");
-}
-
-__device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
-  uint32_t ok = 0;
-  while (!ok) {
-    asm volatile(
-        "{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2; "
-        "selp.u32 %0, 1, 0, p; }"
-        : "=r"(ok)
-        : "r"(smem_u32(bar)), "r"(parity)
-        : "memory");
-  }
-}
-
-__device__ __forceinline__ void bulk_load(void *smem_dst, const void *gmem_src, uint32_t bytes,
-                                          uint64_t *bar) {
-  asm volatile(
-      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
-          smem_u32(smem_dst)),
-      "l"(gmem_src), "r"(bytes), "r"(smem_u32(bar))
-      : "memory");
-}
-
-// Geometry of one (tree, channel) stream of segments, identical in every warp.
-struct SegMap {
-  uint64_t chunk_stride;  // bytes between consecutive tree-local chunks (T * E_b)
-  uint64_t first;         // byte offset of slice j of tree-local chunk 0
-  uint32_t nseg;          // segments per full slice
-  uint32_t kfull;         // tree-local chunks with a full-length slice
-  uint32_t sl_full;       // bytes of a full slice for this channel
-  uint32_t nseg_last;     // segments of the last (short) chunk, incl. a ragged one
-  uint32_t last_len;      // bytes of the last chunk's slice (may end off a 16 B boundary)
-  uint32_t total;         // kfull * nseg + nseg_last
-};
-
-template <int ES>
-__device__ __forceinline__ SegMap seg_map(const LaunchArgs &a, int t, int j) {
-  SegMap m;
-  const uint64_t Eb = static_cast<uint64_t>(a.elems_per_chunk) * ES;
-  const uint64_t SLb = static_cast<uint64_t>(a.slice_elems) * ES;
-  const uint64_t jo = static_cast<uint64_t>(j) * SLb;
-  m.chunk_stride = Eb * a.ntrees;
-  m.first = static_cast<uint64_t>(t) * Eb + jo;
-  m.sl_full = static_cast<uint32_t>(jo < Eb ? min(SLb, Eb - jo) : 0);
-  m.nseg = (m.sl_full + kSeg - 1) / kSeg;
-  const uint32_t K = a.K[t];
-  const uint64_t nbytes = a.count * ES;
-  const uint64_t Ktot = (a.count + a.elems_per_chunk - 1) / a.elems_per_chunk;
-  const uint64_t C = Ktot - 1;  // last global chunk
-  m.kfull = K;
-  m.last_len = 0;
-  m.nseg_last = 0;
-  if (K > 0 && (C % a.ntrees) == static_cast<uint64_t>(t) && nbytes < (C + 1) * Eb) {
-    m.kfull = K - 1;  // this tree carries the short last chunk
-    const uint64_t s0 = C * Eb + jo;
-    m.last_len = static_cast<uint32_t>(s0 < nbytes ? min(SLb, nbytes - s0) : 0);
-    const uint32_t aligned = m.last_len & ~15u;
-    m.nseg_last = (aligned + kSeg - 1) / kSeg + ((m.last_len & 15u) ? 1 : 0);
-  }
-  m.total = m.nseg ? m.kfull * m.nseg + m.nseg_last : m.nseg_last;
-  return m;
-}
-
-__device__ __forceinline__ uint32_t seg_chunk(const SegMap &m, uint32_t G) {
-  if (m.nseg == 0) return m.kfull;
-  const uint32_t k = G / m.nseg;
-  return k < m.kfull ? k : m.kfull;
-}
-
-// byte offset within the buffer and length of segment G; len < 16 marks the
-// ragged sub-vector tail at the very end of the buffer (scalar path, no TMA)
-__device__ __forceinline__ void seg_range(const SegMap &m, uint32_t G, uint64_t *off,
-                                          uint32_t *len) {
-  const uint32_t k = seg_chunk(m, G);
-  const uint32_t s = G - k * m.nseg;
-  const uint64_t base = m.first + static_cast<uint64_t>(k) * m.chunk_stride;
-  if (k < m.kfull) {
-    *off = base + static_cast<uint64_t>(s) * kSeg;
-    *len = min(static_cast<uint32_t>(kSeg), m.sl_full - s * kSeg);
-    return;
-  }
-  const uint32_t aligned = m.last_len & ~15u;
-  const uint32_t full_segs = (aligned + kSeg - 1) / kSeg;
-  if (s < full_segs) {
-    *off = base + static_cast<uint64_t>(s) * kSeg;
-    *len = min(static_cast<uint32_t>(kSeg), aligned - s * kSeg);
-  } else {
-    *off = base + aligned;
-    *len = m.last_len - aligned;  // 1..15 bytes
-  }
-}
-
+// ---- consumer (data) warps -----------------------------------------------------------
 template <int DT, int NIN>
-__device__ __forceinline__ void combine_stage(const char *stage, uint32_t len, char *const *dst,
-                                              int nout, uint64_t off) {
+__device__ __forceinline__ void combine_stage(char *stages, uint32_t seg, int st, uint32_t len,
+                                              char *const *dst, int nout, uint64_t off, int w,
+                                              int W) {
   const int lane = threadIdx.x & 31;
-  for (uint32_t v = lane; v < len / 16; v += 32) {
+  const char *b = stage_ptr(stages, seg, st, 0);
+  for (uint32_t v = w * 32 + lane; v < len / 16; v += W * 32) {
     uint4 x[NIN];
 #pragma unroll
     for (int q = 0; q < NIN; ++q)
-      x[q] = *reinterpret_cast<const uint4 *>(stage + q * kSeg + v * 16);
+      x[q] = *reinterpret_cast<const uint4 *>(b + static_cast<size_t>(q) * seg + v * 16);
     const uint4 r = Combine<DT>::template vec<NIN>(x);
     for (int d = 0; d < nout; ++d) *reinterpret_cast<uint4 *>(dst[d] + off + v * 16) = r;
   }
@@ -491,116 +562,45 @@ __device__ __forceinline__ void combine_scalar(const char *const *src, int nin, 
   char *dd[kMaxIn];
   for (int q = 0; q < nin; ++q) ss[q] = src[q] + off;
   for (int q = 0; q < nout; ++q) dd[q] = dst[q] + off;
-  for (uint32_t e = lane; e < len / ES; e += 32) {
+  for (uint32_t x = lane; x < len / ES; x += 32) {
     switch (nin) {
-      case 1: Combine<DT>::template scalar<1>(ss, dd, nout, e); break;
-      case 2: Combine<DT>::template scalar<2>(ss, dd, nout, e); break;
-      default: Combine<DT>::template scalar<3>(ss, dd, nout, e); break;
+      case 1: Combine<DT>::template scalar<1>(ss, dd, nout, x); break;
+      case 2: Combine<DT>::template scalar<2>(ss, dd, nout, x); break;
+      default: Combine<DT>::template scalar<3>(ss, dd, nout, x); break;
     }
   }
 }
 
 template <int DT>
 __device__ void data_warp(const LaunchArgs &a, const TreeParams &p, int role, int t, int j,
-                          int w, int W, Shared &sh, char *stage_base, uint64_t *bars) {
+                          int w, int W, Shared &sh, char *stages) {
   constexpr int ES = DT == kBFloat16 ? 2 : 4;
   const int lane = threadIdx.x & 31;
-  const uint32_t K = a.K[t];
-  const char *src[kMaxIn];
-  char *dst[kMaxIn];
-  int nin, nout;
-  if (role == kRoleUp) {
-    nin = 1 + p.nchild;
-    for (int q = 0; q < nin; ++q) src[q] = p.up_src[q];
-    dst[0] = p.up_dst;
-    nout = 1;
-    if (p.is_root && a.overlap) {  // C1 turnaround: final straight into the children
-      for (int s = 0; s < p.nchild; ++s) dst[1 + s] = p.child_buf[s];
-      nout += p.nchild;
-    }
-  } else {
-    nin = 1;
-    src[0] = p.buf;
-    for (int s = 0; s < p.nchild; ++s) dst[s] = p.child_buf[s];
-    nout = p.nchild;
-  }
+  const Endpoints e = endpoints(a, p, role);
   const SegMap m = seg_map<ES>(a, t, j);
-  const uint32_t mine = m.total > static_cast<uint32_t>(w)
-                            ? (m.total - w + W - 1) / W : 0;  // segments w, w+W, ...
-  char *my_stages = stage_base + static_cast<size_t>(w) * kStages * kMaxIn * kSeg;
-  uint64_t *my_bars = bars + w * kStages;
-  if (lane == 0) {
-    for (int s = 0; s < kStages; ++s) mbar_init(&my_bars[s]);
-    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-  }
-  __syncwarp();
-
-  uint32_t issued = 0, consumed = 0, done_reported = 0;
-  uint64_t ready = 0;
-  while (consumed < mine) {
-    // issue every segment whose chunk is ready, up to kStages ahead
-    while (issued < mine && issued - consumed < kStages) {
-      const uint32_t G = w + issued * W;
-      const uint32_t k = seg_chunk(m, G);
-      if (k >= ready) {
-        if (issued > consumed) break;  // work is staged: consume it first
-        uint64_t r = 0;
-        if (lane == 0) {
-          do {
-            r = ld_acquire_cta(&sh.ready);
-          } while (r <= k && !*reinterpret_cast<volatile int *>(&sh.abort));
-          // order the generic-proxy acquire before the async-proxy (TMA) reads
-          asm volatile("fence.proxy.async.global;" ::: "memory");
-        }
-        r = __shfl_sync(0xffffffffu, r, 0);
-        if (r <= k) return;  // aborted
-        ready = r;
+  for (uint32_t G = 0; G < m.total; ++G) {
+    const int st = G % kStages;
+    if (!mbar_wait(&sh.full[st], (G / kStages) & 1, &sh.abort)) return;
+    uint64_t off;
+    uint32_t len;
+    seg_range(m, G, &off, &len);
+    if (len >= 16) {
+      switch (e.nin) {
+        case 1: combine_stage<DT, 1>(stages, m.seg, st, len, e.dst, e.nout, off, w, W); break;
+        case 2: combine_stage<DT, 2>(stages, m.seg, st, len, e.dst, e.nout, off, w, W); break;
+        default: combine_stage<DT, 3>(stages, m.seg, st, len, e.dst, e.nout, off, w, W); break;
       }
-      uint64_t off;
-      uint32_t len;
-      seg_range(m, G, &off, &len);
-      if (lane == 0 && len >= 16) {
-        const int st = issued % kStages;
-        char *buf = my_stages + static_cast<size_t>(st) * kMaxIn * kSeg;
-        mbar_expect_tx(&my_bars[st], len * nin);
-        for (int q = 0; q < nin; ++q) bulk_load(buf + q * kSeg, src[q] + off, len, &my_bars[st]);
-      }
-      ++issued;
+    } else if (w == 0) {
+      combine_scalar<DT>(e.src, e.nin, e.dst, e.nout, off, len);
     }
-    // consume the oldest staged segment
-    {
-      const uint32_t G = w + consumed * W;
-      uint64_t off;
-      uint32_t len;
-      seg_range(m, G, &off, &len);
-      const int st = consumed % kStages;
-      if (len >= 16) {
-        mbar_wait(&my_bars[st], (consumed / kStages) & 1);
-        const char *buf = my_stages + static_cast<size_t>(st) * kMaxIn * kSeg;
-        switch (nin) {
-          case 1: combine_stage<DT, 1>(buf, len, dst, nout, off); break;
-          case 2: combine_stage<DT, 2>(buf, len, dst, nout, off); break;
-          default: combine_stage<DT, 3>(buf, len, dst, nout, off); break;
-        }
-      } else {
-        combine_scalar<DT>(src, nin, dst, nout, off, len);
-      }
-      __syncwarp();  // every lane is done with the stage and has issued its stores
-      ++consumed;
-      const uint32_t d = consumed < mine ? seg_chunk(m, w + consumed * W) : K;
-      if (d > done_reported) {
-        if (lane == 0) st_release_cta(&sh.done[w], d);
-        done_reported = d;
-      }
-    }
+    __syncwarp();  // all lanes done with the stage and their stores issued
+    if (lane == 0) mbar_arrive(&sh.empty[st]);
   }
-  if (done_reported < K && lane == 0) st_release_cta(&sh.done[w], K);
 }
 
 template <int DT, bool SYS>
 __global__ void __launch_bounds__(kMaxThreads) tree_allreduce_kernel(const LaunchArgs a) {
   __shared__ Shared sh;
-  __shared__ uint64_t bars[kMaxDataWarps * kStages];
   extern __shared__ __align__(128) char stages[];
   const Task task = a.tasks[blockIdx.x];
   const TreeParams &p = a.params[task.local_rank * a.ntrees + task.tree];
@@ -611,15 +611,19 @@ __global__ void __launch_bounds__(kMaxThreads) tree_allreduce_kernel(const Launc
   }
   const int W = (blockDim.x >> 5) - 1;
   if (threadIdx.x == 0) {
-    sh.ready = 0;
+    for (int s = 0; s < kStages; ++s) {
+      mbar_init(&sh.full[s], 1);
+      mbar_init(&sh.empty[s], W);
+    }
     sh.abort = 0;
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
-  if (threadIdx.x < kMaxDataWarps) sh.done[threadIdx.x] = 0;
   __syncthreads();
+  constexpr int ES = DT == kBFloat16 ? 2 : 4;
   if (warp == 0)
-    control_warp<SYS>(a, p, task.role, task.tree, task.channel, W, sh);
+    control_warp<ES, SYS>(a, p, task.role, task.tree, task.channel, sh, stages);
   else
-    data_warp<DT>(a, p, task.role, task.tree, task.channel, warp - 1, W, sh, stages, bars);
+    data_warp<DT>(a, p, task.role, task.tree, task.channel, warp - 1, W, sh, stages);
 }
 
 struct GateArgs {
@@ -646,13 +650,11 @@ __global__ void gate_kernel(const GateArgs g) {
   }
 }
 
-size_t stage_bytes(int threads) {
-  return static_cast<size_t>(threads / 32 - 1) * kStages * kMaxIn * kSeg;
-}
+size_t stage_bytes(uint32_t seg) { return static_cast<size_t>(kStages) * kMaxIn * seg; }
 
 template <int DT, bool SYS>
 int launch_t(const LaunchArgs &a, int grid, int threads, cudaStream_t s) {
-  const size_t smem = stage_bytes(threads);
+  const size_t smem = stage_bytes(a.seg_bytes);
   cudaError_t e = cudaFuncSetAttribute(tree_allreduce_kernel<DT, SYS>,
                                        cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        static_cast<int>(smem));
@@ -671,7 +673,7 @@ const void *kernel_ptr() {
 int launch_tree_allreduce(const LaunchArgs &args, int dtype, bool sys_scope, int grid,
                           int threads, void *stream) {
   if (threads > kMaxThreads || threads < 64 || threads % 32 ||
-      threads / 32 - 1 > kMaxDataWarps)
+      threads / 32 - 1 > kMaxDataWarps || args.seg_bytes < 16 || args.seg_bytes % 16)
     return cudaErrorInvalidValue;
   cudaStream_t s = static_cast<cudaStream_t>(stream);
   switch (dtype) {
@@ -709,7 +711,8 @@ int launch_gate(const uint64_t *const *counters, const uint64_t *targets, int n,
   return static_cast<int>(cudaGetLastError());
 }
 
-int query_max_blocks_per_sm(int dtype, bool sys_scope, int threads, int *blocks) {
+int query_max_blocks_per_sm(int dtype, bool sys_scope, int threads, uint32_t seg_bytes,
+                            int *blocks) {
   const void *fn = nullptr;
   switch (dtype) {
     case kInt32:
@@ -722,7 +725,7 @@ int query_max_blocks_per_sm(int dtype, bool sys_scope, int threads, int *blocks)
       fn = sys_scope ? kernel_ptr<kBFloat16, true>() : kernel_ptr<kBFloat16, false>();
       break;
   }
-  const size_t smem = stage_bytes(threads);
+  const size_t smem = stage_bytes(seg_bytes);
   cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        static_cast<int>(smem));
   if (e != cudaSuccess) return static_cast<int>(e);
