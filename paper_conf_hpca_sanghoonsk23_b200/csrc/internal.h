@@ -69,6 +69,7 @@ struct TreeParams {
 };
 
 enum Role { kRoleUp = 0, kRoleDown = 1 };
+enum Datapath { kDatapathLsu = 0, kDatapathTma = 1 };
 
 enum { kAllChannels = -1 };  // a pulled leaf's single task covers every channel
 
@@ -90,7 +91,7 @@ struct LaunchArgs {
   uint32_t K[kMaxTrees];      // tree-local chunk counts
   uint64_t base[kMaxTrees];   // counter base of this call per tree
   int overlap;                // 1 = C1, 0 = B
-  int pad0;
+  int datapath;               // kDatapathLsu (register-staged) or kDatapathTma
   uint64_t timeout_ns;        // watchdog
   int *err;                   // mapped host word; nonzero = abort
   uint64_t *trace;            // optional landing trace
@@ -104,7 +105,7 @@ int launch_tree_allreduce(const LaunchArgs &args, int dtype, bool sys_scope, int
 constexpr int kMaxGateCounters = 128;
 int launch_gate(const uint64_t *const *counters, const uint64_t *targets, int n, int *err,
                 uint64_t timeout_ns, bool sys_scope, void *stream);
-int query_max_blocks_per_sm(int dtype, bool sys_scope, int threads, uint32_t seg_bytes,
-                            int *blocks);
+int query_max_blocks_per_sm(int dtype, bool sys_scope, int threads, int datapath,
+                            uint32_t seg_bytes, int *blocks);
 
 }  // namespace ccube

@@ -171,6 +171,7 @@ struct Comm {
   std::map<std::pair<int, int>, TaskTable> tasks;  // (channels, overlap)
   int transport = CCUBE_TRANSPORT_AUTO;
   uint32_t seg_bytes = 16384;  // TMA stage bytes per source
+  int datapath = kDatapathLsu;
   bool sys_scope = false;
   uint64_t timeout_ns = 10000ull * 1000000ull;
   int sm_count = 0;
@@ -488,10 +489,12 @@ ccube_result_t allreduce_impl(void *const *bufs, size_t count, ccube_dtype_t dty
 
   // all CTAs spin on each other: they must be co-resident
   const int cta_threads = g.threads + 32;  // data warps + the control warp
-  auto key = std::make_pair((int)dtype, cta_threads * 1024 + (int)(g.seg_bytes >> 4));
+  auto key = std::make_pair((int)dtype * 2 + g.datapath,
+                            cta_threads * 1024 + (int)(g.seg_bytes >> 4));
   if (!g.max_blocks.count(key)) {
     int b = 0;
-    const int rc = query_max_blocks_per_sm(dtype, g.sys_scope, cta_threads, g.seg_bytes, &b);
+    const int rc =
+        query_max_blocks_per_sm(dtype, g.sys_scope, cta_threads, g.datapath, g.seg_bytes, &b);
     if (rc != cudaSuccess)
       return fail(CCUBE_ERR_CUDA, "occupancy query failed: %s",
                   cudaGetErrorString(static_cast<cudaError_t>(rc)));
@@ -526,6 +529,7 @@ ccube_result_t allreduce_impl(void *const *bufs, size_t count, ccube_dtype_t dty
   a.trace = g.trace;
   a.trace_kmax = static_cast<uint32_t>(g.trace_kmax);
   a.seg_bytes = g.seg_bytes;
+  a.datapath = g.datapath;
   a.params = R->d_params;
 
   TaskTable *tt = nullptr;
@@ -659,7 +663,7 @@ ccube_result_t ccube_init(const ccube_world_t *world, ccube_tree_kind_t tree_kin
   if (channels < 0 || channels > CCUBE_MAX_CHANNELS)
     return fail(CCUBE_ERR_INVALID_ARG, "CCUBE_CHANNELS %d out of range", channels);
   CC_TRY(check_chunk(chunk_bytes));
-  int threads = env_int("CCUBE_THREADS", 256);
+  int threads = env_int("CCUBE_THREADS", 512);
   if (threads < 32 || threads > 512 || threads % 32)
     return fail(CCUBE_ERR_INVALID_ARG, "CCUBE_THREADS %d out of range [32, 512]", threads);
   const int transport = env_int("CCUBE_TRANSPORT", CCUBE_TRANSPORT_AUTO);
@@ -680,6 +684,7 @@ ccube_result_t ccube_init(const ccube_world_t *world, ccube_tree_kind_t tree_kin
   g.channels = channels;
   g.threads = threads;
   g.transport = transport;
+  g.datapath = env_int("CCUBE_DATAPATH_TMA", 0) ? kDatapathTma : kDatapathLsu;
   g.seg_bytes = static_cast<uint32_t>(env_int("CCUBE_SEG_BYTES", 16384));
   if (g.seg_bytes < 1024 || g.seg_bytes > 16384 || g.seg_bytes % 1024) {
     g = Comm();

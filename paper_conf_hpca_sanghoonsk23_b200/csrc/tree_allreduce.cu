@@ -382,10 +382,22 @@ __device__ __forceinline__ Endpoints endpoints(const LaunchArgs &a, const TreePa
 }
 
 struct Shared {
-  uint64_t full[kStages];   // producer -> consumers: stage loaded (TMA complete_tx)
-  uint64_t empty[kStages];  // consumers -> producer: stage consumed, stores issued
+  uint64_t full[kStages];   // TMA path: producer -> consumers, stage loaded (complete_tx)
+  uint64_t empty[kStages];  // TMA path: consumers -> producer, stage consumed
+  uint64_t ready;           // LSU path: chunks whose inputs are available (control -> data)
+  uint64_t done[kMaxDataWarps];  // LSU path: chunks finished by data warp w (data -> control)
   int abort;
 };
+
+// CTA-scope release/acquire on shared memory (control <-> data warps)
+__device__ __forceinline__ void st_release_cta(uint64_t *p, uint64_t v) {
+  asm volatile("st.release.cta.shared.u64 [%0], %1;" ::"r"(smem_u32(p)), "l"(v) : "memory");
+}
+__device__ __forceinline__ uint64_t ld_acquire_cta(const uint64_t *p) {
+  uint64_t v;
+  asm volatile("ld.acquire.cta.shared.u64 %0, [%1];" : "=l"(v) : "r"(smem_u32(p)) : "memory");
+  return v;
+}
 
 __device__ __forceinline__ char *stage_ptr(char *stages, uint32_t seg, int st, int q) {
   return stages + (static_cast<size_t>(st) * kMaxIn + q) * seg;
@@ -414,9 +426,27 @@ __device__ __forceinline__ void publish(const LaunchArgs &a, const TreeParams &p
   }
 }
 
+// Leaf completion: the kernel completes only once the whole result has landed.
+template <bool SYS>
+__device__ __forceinline__ void leaf_wait(const LaunchArgs &a, const TreeParams &p, int role,
+                                          int t, int j) {
+  const int stride = j * kFlagStrideU64;
+  const uint64_t target = a.base[t] + a.K[t];
+  if (role == kRoleUp && !p.is_root && p.nchild == 0 && (threadIdx.x & 31) == 0) {
+    Watch wd;
+    watch_reset(wd);
+    while (ld_acquire<SYS>(p.enq + stride) < target) {
+      if (!watch_tick(wd, a, target, 0)) {
+        st_relaxed<SYS>(p.enq + stride, ~0ull);
+        return;
+      }
+    }
+  }
+}
+
 template <int ES, bool SYS>
-__device__ void control_warp(const LaunchArgs &a, const TreeParams &p, int role, int t, int j,
-                             Shared &sh, char *stages) {
+__device__ void control_warp_tma(const LaunchArgs &a, const TreeParams &p, int role, int t, int j,
+                                 Shared &sh, char *stages) {
   const int lane = threadIdx.x & 31;
   const uint32_t K = a.K[t];
   const uint64_t base = a.base[t];
@@ -502,16 +532,7 @@ __device__ void control_warp(const LaunchArgs &a, const TreeParams &p, int role,
       return;
     }
   }
-  // a leaf's kernel completes only once the whole result has landed in its buffer
-  if (role == kRoleUp && !p.is_root && p.nchild == 0 && lane == 0) {
-    watch_reset(wd);
-    while (ld_acquire<SYS>(p.enq + stride) < base + K) {
-      if (!watch_tick(wd, a, base + K, 0)) {
-        st_relaxed<SYS>(p.enq + stride, ~0ull);
-        return;
-      }
-    }
-  }
+  leaf_wait<SYS>(a, p, role, t, j);
 }
 
 // A leaf on a PULL edge: its input already sits where the parent reads it.  One
@@ -572,8 +593,8 @@ __device__ __forceinline__ void combine_scalar(const char *const *src, int nin, 
 }
 
 template <int DT>
-__device__ void data_warp(const LaunchArgs &a, const TreeParams &p, int role, int t, int j,
-                          int w, int W, Shared &sh, char *stages) {
+__device__ void data_warp_tma(const LaunchArgs &a, const TreeParams &p, int role, int t, int j,
+                              int w, int W, Shared &sh, char *stages) {
   constexpr int ES = DT == kBFloat16 ? 2 : 4;
   const int lane = threadIdx.x & 31;
   const Endpoints e = endpoints(a, p, role);
@@ -598,6 +619,208 @@ __device__ void data_warp(const LaunchArgs &a, const TreeParams &p, int role, in
   }
 }
 
+// ---- LSU path (default): register-staged data warps ------------------------------
+// The control warp polls upstream and publishes "chunks ready" in shared memory;
+// each data warp streams its items — 16-byte vectors w*32+lane, stepping W*32,
+// across the concatenated slices of all chunks — in rounds of U vectors per
+// lane per source.  A round may span chunk boundaries (it only needs every lane's
+// chunk to be ready), so loads stay in flight across chunks; per-warp "done"
+// counters (the chunk of the warp's next item) let the control warp publish
+// downstream.
+template <bool SYS>
+__device__ void control_warp_lsu(const LaunchArgs &a, const TreeParams &p, int role, int t, int j,
+                                 int W, Shared &sh) {
+  const int lane = threadIdx.x & 31;
+  const uint32_t K = a.K[t];
+  const uint64_t base = a.base[t];
+  const int stride = j * kFlagStrideU64;
+  const uint64_t *up = nullptr;
+  if (role == kRoleUp) {
+    if (lane < p.nchild) up = p.head_in[lane] + stride;
+  } else if (lane == 0) {
+    up = p.enq + stride;
+  }
+  const bool hold_all = role == kRoleDown && p.is_root;  // B-mode root (Obs #1)
+  uint64_t ready = (role == kRoleUp && p.nchild == 0) ? K : 0;  // a leaf's input is ready
+  if (lane == 0) st_release_cta(&sh.ready, ready);
+  uint32_t pub = 0;
+  Watch wd;
+  watch_reset(wd);
+  while (pub < K) {
+    bool moved = false;
+    if (ready < K) {
+      uint64_t v = up ? ld_acquire<SYS>(up) : ~0ull;
+      v = warp_min(v);
+      uint64_t r = v > base ? v - base : 0;
+      if (r > K) r = K;
+      if (hold_all && r < K) r = 0;
+      if (r > ready) {
+        __syncwarp();  // every lane's acquire happens before lane 0's release below
+        ready = r;
+        if (lane == 0) st_release_cta(&sh.ready, ready);
+        moved = true;
+      }
+    }
+    uint64_t d = lane < W ? ld_acquire_cta(&sh.done[lane]) : ~0ull;
+    d = warp_min(d);
+    if (d > pub) {
+      __syncwarp();
+      if (lane == 0) publish<SYS>(a, p, role, t, j, pub, static_cast<uint32_t>(d), base);
+      pub = static_cast<uint32_t>(d);
+      moved = true;
+    }
+    if (moved) {
+      watch_reset(wd);
+    } else if (!watch_tick(wd, a, base + ready + 1, base + pub)) {
+      if (lane == 0) {
+        *reinterpret_cast<volatile int *>(&sh.abort) = 1;
+        st_relaxed<SYS>(p.enq + stride, ~0ull);  // release gradient-queue waiters
+      }
+      return;
+    }
+  }
+  leaf_wait<SYS>(a, p, role, t, j);
+}
+
+// Item geometry of one (tree, channel) stream in 16-byte vectors.
+struct VecMap {
+  uint64_t first;         // byte offset of slice j of tree-local chunk 0
+  uint64_t chunk_stride;  // bytes between consecutive tree-local chunks
+  uint32_t nv_full;       // vectors of a full slice
+  uint32_t nv_last;       // vectors of the short last chunk's slice (if this tree has it)
+  uint32_t kfull;         // chunks with a full slice (K or K-1)
+  uint32_t ragged;        // bytes after the last whole vector of the buffer (0..15)
+};
+
+template <int ES>
+__device__ __forceinline__ VecMap vec_map(const LaunchArgs &a, int t, int j) {
+  const SegMap s = seg_map<ES>(a, t, j);
+  VecMap m;
+  m.first = s.first;
+  m.chunk_stride = s.chunk_stride;
+  m.nv_full = s.sl_full / 16;
+  m.kfull = s.kfull;
+  m.nv_last = s.last_len / 16;
+  m.ragged = s.last_len & 15u;
+  return m;
+}
+
+// Normalise (k, v) so that v < vectors(k), or k == K (past the end).
+__device__ __forceinline__ void vec_norm(const VecMap &m, uint32_t K, uint32_t &k, uint32_t &v) {
+  while (k < K) {
+    const uint32_t n = k < m.kfull ? m.nv_full : m.nv_last;
+    if (v < n) return;
+    v -= n;
+    ++k;
+  }
+}
+
+template <int DT, int NIN, int NOUT, int U>
+__device__ void lsu_stream(const LaunchArgs &a, const Endpoints &e, const VecMap &m, uint32_t K,
+                           int w, int W, Shared &sh, bool do_ragged) {
+  const int lane = threadIdx.x & 31;
+  const uint32_t step = static_cast<uint32_t>(W) * 32;
+  uint32_t k = 0, v = static_cast<uint32_t>(w) * 32 + lane;
+  vec_norm(m, K, k, v);
+  uint64_t ready = 0;
+  uint32_t done_reported = 0;
+  bool ragged_left = do_ragged;
+  while (true) {
+    const uint32_t k0 = __shfl_sync(0xffffffffu, k, 0);
+    if (k0 >= K) break;
+    if (k0 >= ready) {
+      uint64_t r = 0;
+      if (lane == 0) {
+        do {
+          r = ld_acquire_cta(&sh.ready);
+        } while (r <= k0 && !*reinterpret_cast<volatile int *>(&sh.abort));
+      }
+      r = __shfl_sync(0xffffffffu, r, 0);
+      if (r <= k0) return;  // aborted
+      ready = r;
+    }
+    uint32_t kk[U], vv[U];
+    uint32_t ck = k, cv = v;
+    int rounds = 0;
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      kk[u] = ck;
+      vv[u] = cv;
+      const uint32_t kmax = __reduce_max_sync(0xffffffffu, ck < K ? ck : 0);
+      const bool any = __any_sync(0xffffffffu, ck < K);
+      if (rounds == u && any && kmax < ready) {
+        rounds = u + 1;
+        cv += step;
+        vec_norm(m, K, ck, cv);
+      }
+    }
+    uint4 x[U][NIN];
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      if (u < rounds && kk[u] < K) {
+        const uint64_t off = m.first + kk[u] * m.chunk_stride + static_cast<uint64_t>(vv[u]) * 16;
+#pragma unroll
+        for (int q = 0; q < NIN; ++q) x[u][q] = __ldcg(reinterpret_cast<const uint4 *>(e.src[q] + off));
+      }
+    }
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      if (u < rounds && kk[u] < K) {
+        const uint64_t off = m.first + kk[u] * m.chunk_stride + static_cast<uint64_t>(vv[u]) * 16;
+        const uint4 r = Combine<DT>::template vec<NIN>(x[u]);
+#pragma unroll
+        for (int q = 0; q < NOUT; ++q) *reinterpret_cast<uint4 *>(e.dst[q] + off) = r;
+      }
+    }
+    k = ck;
+    v = cv;
+    uint32_t d = __shfl_sync(0xffffffffu, k, 0);  // lane 0 holds the warp's smallest item
+    if (ragged_left && d >= K) d = K - 1;
+    if (d > done_reported) {
+      __syncwarp();
+      if (lane == 0) st_release_cta(&sh.done[w], d);
+      done_reported = d;
+    }
+  }
+  if (ragged_left) {  // sub-vector tail at the end of the buffer (last chunk, now ready)
+    const uint64_t off = m.first + static_cast<uint64_t>(m.kfull) * m.chunk_stride +
+                         static_cast<uint64_t>(m.nv_last) * 16;
+    combine_scalar<DT>(e.src, NIN, e.dst, NOUT, off, m.ragged);
+  }
+  __syncwarp();
+  if (lane == 0) st_release_cta(&sh.done[w], K);
+}
+
+template <int DT, int NIN>
+__device__ __forceinline__ void lsu_nout(const LaunchArgs &a, const Endpoints &e, const VecMap &m,
+                                         uint32_t K, int w, int W, Shared &sh, bool rag) {
+  constexpr int U = NIN == 1 ? 8 : (NIN == 2 ? 6 : 4);
+  switch (e.nout) {
+    case 1: lsu_stream<DT, NIN, 1, U>(a, e, m, K, w, W, sh, rag); break;
+    case 2: lsu_stream<DT, NIN, 2, U>(a, e, m, K, w, W, sh, rag); break;
+    default: lsu_stream<DT, NIN, 3, U>(a, e, m, K, w, W, sh, rag); break;
+  }
+}
+
+template <int DT>
+__device__ void data_warp_lsu(const LaunchArgs &a, const TreeParams &p, int role, int t, int j,
+                              int w, int W, Shared &sh) {
+  constexpr int ES = DT == kBFloat16 ? 2 : 4;
+  const Endpoints e = endpoints(a, p, role);
+  const VecMap m = vec_map<ES>(a, t, j);
+  const uint32_t K = a.K[t];
+  const bool rag = w == 0 && m.ragged != 0;
+  if (e.nout == 0) {  // nothing to write (cannot happen for scheduled tasks)
+    if ((threadIdx.x & 31) == 0) st_release_cta(&sh.done[w], K);
+    return;
+  }
+  switch (e.nin) {
+    case 1: lsu_nout<DT, 1>(a, e, m, K, w, W, sh, rag); break;
+    case 2: lsu_nout<DT, 2>(a, e, m, K, w, W, sh, rag); break;
+    default: lsu_nout<DT, 3>(a, e, m, K, w, W, sh, rag); break;
+  }
+}
+
 template <int DT, bool SYS>
 __global__ void __launch_bounds__(kMaxThreads) tree_allreduce_kernel(const LaunchArgs a) {
   __shared__ Shared sh;
@@ -615,15 +838,24 @@ __global__ void __launch_bounds__(kMaxThreads) tree_allreduce_kernel(const Launc
       mbar_init(&sh.full[s], 1);
       mbar_init(&sh.empty[s], W);
     }
+    sh.ready = 0;
     sh.abort = 0;
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
+  if (threadIdx.x < kMaxDataWarps) sh.done[threadIdx.x] = 0;
   __syncthreads();
   constexpr int ES = DT == kBFloat16 ? 2 : 4;
-  if (warp == 0)
-    control_warp<ES, SYS>(a, p, task.role, task.tree, task.channel, sh, stages);
-  else
-    data_warp<DT>(a, p, task.role, task.tree, task.channel, warp - 1, W, sh, stages);
+  if (a.datapath == kDatapathTma) {
+    if (warp == 0)
+      control_warp_tma<ES, SYS>(a, p, task.role, task.tree, task.channel, sh, stages);
+    else
+      data_warp_tma<DT>(a, p, task.role, task.tree, task.channel, warp - 1, W, sh, stages);
+  } else {
+    if (warp == 0)
+      control_warp_lsu<SYS>(a, p, task.role, task.tree, task.channel, W, sh);
+    else
+      data_warp_lsu<DT>(a, p, task.role, task.tree, task.channel, warp - 1, W, sh);
+  }
 }
 
 struct GateArgs {
@@ -650,11 +882,13 @@ __global__ void gate_kernel(const GateArgs g) {
   }
 }
 
-size_t stage_bytes(uint32_t seg) { return static_cast<size_t>(kStages) * kMaxIn * seg; }
+size_t stage_bytes(int datapath, uint32_t seg) {
+  return datapath == kDatapathTma ? static_cast<size_t>(kStages) * kMaxIn * seg : 0;
+}
 
 template <int DT, bool SYS>
 int launch_t(const LaunchArgs &a, int grid, int threads, cudaStream_t s) {
-  const size_t smem = stage_bytes(a.seg_bytes);
+  const size_t smem = stage_bytes(a.datapath, a.seg_bytes);
   cudaError_t e = cudaFuncSetAttribute(tree_allreduce_kernel<DT, SYS>,
                                        cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        static_cast<int>(smem));
@@ -711,8 +945,8 @@ int launch_gate(const uint64_t *const *counters, const uint64_t *targets, int n,
   return static_cast<int>(cudaGetLastError());
 }
 
-int query_max_blocks_per_sm(int dtype, bool sys_scope, int threads, uint32_t seg_bytes,
-                            int *blocks) {
+int query_max_blocks_per_sm(int dtype, bool sys_scope, int threads, int datapath,
+                            uint32_t seg_bytes, int *blocks) {
   const void *fn = nullptr;
   switch (dtype) {
     case kInt32:
@@ -725,7 +959,7 @@ int query_max_blocks_per_sm(int dtype, bool sys_scope, int threads, uint32_t seg
       fn = sys_scope ? kernel_ptr<kBFloat16, true>() : kernel_ptr<kBFloat16, false>();
       break;
   }
-  const size_t smem = stage_bytes(seg_bytes);
+  const size_t smem = stage_bytes(datapath, seg_bytes);
   cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        static_cast<int>(smem));
   if (e != cudaSuccess) return static_cast<int>(e);

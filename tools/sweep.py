@@ -28,6 +28,7 @@ def main():
     p.add_argument("--iters", type=int, default=20)
     p.add_argument("--transport", default="auto")
     p.add_argument("--seg", default="16384")
+    p.add_argument("--tma", default="0")
     p.add_argument("--bytes", type=int, default=0, help="override buffer bytes per rank")
     a = p.parse_args()
     tdt = {"float32": torch.float32, "bfloat16": torch.bfloat16, "int32": torch.int32}[a.dtype]
@@ -37,11 +38,12 @@ def main():
     bufs = [torch.randn(count, device="cuda").to(tdt) for _ in range(P)]
     flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
     s = torch.cuda.Stream()
-    for tree, ov, ch, th, cb, tp, sg in itertools.product(
+    for tree, ov, ch, th, cb, tp, sg, tma in itertools.product(
             a.trees.split(","), a.overlap.split(","), a.channels.split(","), a.threads.split(","),
-            a.chunks.split(","), a.transport.split(","), a.seg.split(",")):
+            a.chunks.split(","), a.transport.split(","), a.seg.split(","), a.tma.split(",")):
         try:
             os.environ["CCUBE_SEG_BYTES"] = sg
+            os.environ["CCUBE_DATAPATH_TMA"] = tma
             ccube.init_loopback(P, tree, int(cb))
             ccube.set_channels(int(ch))
             ccube.set_threads(int(th))
@@ -62,7 +64,7 @@ def main():
             nbytes = count * es
             busbw = nbytes / (med / 1e3) / 1e9 * 2 * (P - 1) / P
             hbm = 2 * P * nbytes / (med / 1e3) / 1e9
-            print(json.dumps({"tree": tree, "transport": tp, "seg": int(sg), "overlap": int(ov),
+            print(json.dumps({"tree": tree, "tma": int(tma), "transport": tp, "seg": int(sg), "overlap": int(ov),
                               "channels_used": ccube.get_info()["channels"], "channels": int(ch),
                               "threads": int(th), "chunk": int(cb), "ms": round(med, 4),
                               "busbw": round(busbw, 1), "hbm_algo_gbs": round(hbm, 1)}),
