@@ -728,15 +728,17 @@ __device__ void lsu_stream(const LaunchArgs &a, const Endpoints &e, const VecMap
   while (true) {
     const uint32_t k0 = __shfl_sync(0xffffffffu, k, 0);
     if (k0 >= K) break;
-    if (k0 >= ready) {
+    // every lane's next item must be in a ready chunk before a round can start
+    const uint32_t kneed = __reduce_max_sync(0xffffffffu, k < K ? k : 0);
+    if (kneed >= ready) {
       uint64_t r = 0;
       if (lane == 0) {
         do {
           r = ld_acquire_cta(&sh.ready);
-        } while (r <= k0 && !*reinterpret_cast<volatile int *>(&sh.abort));
+        } while (r <= kneed && !*reinterpret_cast<volatile int *>(&sh.abort));
       }
       r = __shfl_sync(0xffffffffu, r, 0);
-      if (r <= k0) return;  // aborted
+      if (r <= kneed) return;  // aborted
       ready = r;
     }
     uint32_t kk[U], vv[U];
@@ -782,7 +784,17 @@ __device__ void lsu_stream(const LaunchArgs &a, const Endpoints &e, const VecMap
       done_reported = d;
     }
   }
-  if (ragged_left) {  // sub-vector tail at the end of the buffer (last chunk, now ready)
+  if (ragged_left) {  // sub-vector tail at the end of the buffer (in the last chunk)
+    if (ready < K) {
+      uint64_t r = 0;
+      if (lane == 0) {
+        do {
+          r = ld_acquire_cta(&sh.ready);
+        } while (r < K && !*reinterpret_cast<volatile int *>(&sh.abort));
+      }
+      r = __shfl_sync(0xffffffffu, r, 0);
+      if (r < K) return;  // aborted
+    }
     const uint64_t off = m.first + static_cast<uint64_t>(m.kfull) * m.chunk_stride +
                          static_cast<uint64_t>(m.nv_last) * 16;
     combine_scalar<DT>(e.src, NIN, e.dst, NOUT, off, m.ragged);
