@@ -663,7 +663,7 @@ ccube_result_t ccube_init(const ccube_world_t *world, ccube_tree_kind_t tree_kin
   if (channels < 0 || channels > CCUBE_MAX_CHANNELS)
     return fail(CCUBE_ERR_INVALID_ARG, "CCUBE_CHANNELS %d out of range", channels);
   CC_TRY(check_chunk(chunk_bytes));
-  int threads = env_int("CCUBE_THREADS", 512);
+  int threads = env_int("CCUBE_THREADS", 256);
   if (threads < 32 || threads > 512 || threads % 32)
     return fail(CCUBE_ERR_INVALID_ARG, "CCUBE_THREADS %d out of range [32, 512]", threads);
   const int transport = env_int("CCUBE_TRANSPORT", CCUBE_TRANSPORT_AUTO);

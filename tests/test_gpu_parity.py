@@ -70,7 +70,7 @@ def test_parity_small(comm, P, kind, dtype, overlap, transport):
 def test_parity_channels(comm, channels):
     """Channel slices need not divide the chunk (0 = auto: as many as fit)."""
     chunk = 16 * 1024 * 3
-    comm(8, "double", chunk, channels=channels)
+    comm(8, "double", chunk, channels=channels, threads=256)
     count = 5 * chunk // 4 + 1001
     xs, outs = _run(8, "double", "float32", count, chunk)
     ref = oar.reference(xs, "double", chunk, "float32")[0]
