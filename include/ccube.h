@@ -152,8 +152,8 @@ CCUBE_API ccube_result_t ccube_gradq_wait_local(int local_rank, int layer_id, vo
 CCUBE_API ccube_result_t ccube_set_overlap(int on);
 
 /* Channels J per tree (CTA slices of every chunk); all ranks must agree.  0 = the
- * default (CCUBE_CHANNELS env or 8).  `threads` = data threads per CTA (32..512,
- * multiple of 32; CCUBE_THREADS env, default 512); each CTA adds one control warp. */
+ * default (CCUBE_CHANNELS env or 8).  `threads` = data threads per CTA (32..256,
+ * multiple of 32; CCUBE_THREADS env, default 256); each CTA adds one control warp. */
 CCUBE_API ccube_result_t ccube_set_channels(int channels);
 CCUBE_API ccube_result_t ccube_set_threads(int threads);
 

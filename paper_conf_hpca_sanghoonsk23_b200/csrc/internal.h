@@ -85,7 +85,7 @@ struct LaunchArgs {
   const TreeParams *params;   // [local_rank * ntrees + tree]
   uint64_t count;             // elements
   uint32_t elems_per_chunk;   // E
-  uint32_t slice_elems;       // E / J
+  uint32_t pad_slice;         // (unused) channel slices are derived in-kernel, see seg_map
   uint32_t ntrees;
   uint32_t nchannels;
   uint32_t K[kMaxTrees];      // tree-local chunk counts

@@ -506,14 +506,11 @@ ccube_result_t allreduce_impl(void *const *bufs, size_t count, ccube_dtype_t dty
     J = 1;
     while (J < CCUBE_MAX_CHANNELS && count_tasks(J + 1, g.overlap) <= cap) ++J;
   }
-  const uint64_t VE = 16 / es;
-  const uint64_t SL = ((E + J - 1) / J + VE - 1) / VE * VE;  // slice: 16 B multiple
 
   LaunchArgs a;
   memset(&a, 0, sizeof a);
   a.count = count;
   a.elems_per_chunk = static_cast<uint32_t>(E);
-  a.slice_elems = static_cast<uint32_t>(SL);
   a.ntrees = g.ntrees;
   a.nchannels = J;
   if (g.ntrees == 1) {
@@ -664,8 +661,8 @@ ccube_result_t ccube_init(const ccube_world_t *world, ccube_tree_kind_t tree_kin
     return fail(CCUBE_ERR_INVALID_ARG, "CCUBE_CHANNELS %d out of range", channels);
   CC_TRY(check_chunk(chunk_bytes));
   int threads = env_int("CCUBE_THREADS", 256);
-  if (threads < 32 || threads > 512 || threads % 32)
-    return fail(CCUBE_ERR_INVALID_ARG, "CCUBE_THREADS %d out of range [32, 512]", threads);
+  if (threads < 32 || threads > 256 || threads % 32)
+    return fail(CCUBE_ERR_INVALID_ARG, "CCUBE_THREADS %d out of range [32, 256]", threads);
   const int transport = env_int("CCUBE_TRANSPORT", CCUBE_TRANSPORT_AUTO);
   if (transport < CCUBE_TRANSPORT_AUTO || transport > CCUBE_TRANSPORT_PULL)
     return fail(CCUBE_ERR_INVALID_ARG, "CCUBE_TRANSPORT %d out of range", transport);
@@ -867,8 +864,8 @@ ccube_result_t ccube_set_channels(int channels) {
 ccube_result_t ccube_set_threads(int threads) {
   std::lock_guard<std::mutex> lk(g_mu);
   if (!g.init) return fail(CCUBE_ERR_NOT_INITIALIZED, "ccube_init has not been called");
-  if (threads < 32 || threads > 512 || threads % 32)
-    return fail(CCUBE_ERR_INVALID_ARG, "threads %d out of range [32, 512] (multiple of 32)",
+  if (threads < 32 || threads > 256 || threads % 32)
+    return fail(CCUBE_ERR_INVALID_ARG, "threads %d out of range [32, 256] (multiple of 32)",
                 threads);
   g.threads = threads;
   return CCUBE_SUCCESS;

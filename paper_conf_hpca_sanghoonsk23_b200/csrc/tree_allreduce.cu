@@ -36,8 +36,9 @@
 namespace ccube {
 namespace {
 
-constexpr int kMaxThreads = 544;  // up to 16 data warps + the control warp
-constexpr int kMaxDataWarps = 16;
+constexpr int kMaxThreads = 288;  // up to 8 data warps + the control warp
+constexpr int kMaxDataWarps = 8;
+constexpr int kMinBlocksPerSm = 2;  // two CTAs per SM: <= 112 registers per thread
 
 __device__ __forceinline__ uint64_t globaltimer() {
   uint64_t t;
@@ -283,7 +284,12 @@ __device__ __forceinline__ void bulk_load(void *smem_dst, const void *gmem_src, 
 
 // ---- segment geometry --------------------------------------------------------------
 // A CTA's work for (tree t, channel j) is slice j of every tree-local chunk, cut
-// into segments of at most a.seg_bytes per source, processed in order G = 0, 1, ...
+// into segments (TMA path) or blocks (LSU path) of `seg` bytes, taken in order.
+// Channel slices are made of whole kUnit-byte units: channel j owns units
+// [j*n/J, (j+1)*n/J) of the n units of a chunk, so every slice (except at the
+// chunk end) is a multiple of the LSU block size and no lane idles.
+constexpr uint32_t kUnit = 2048;
+
 struct SegMap {
   uint64_t chunk_stride;  // bytes between consecutive tree-local chunks (T * E_b)
   uint64_t first;         // byte offset of slice j of tree-local chunk 0
@@ -297,15 +303,16 @@ struct SegMap {
 };
 
 template <int ES>
-__device__ __forceinline__ SegMap seg_map(const LaunchArgs &a, int t, int j) {
+__device__ __forceinline__ SegMap seg_map(const LaunchArgs &a, int t, int j, uint32_t seg) {
   SegMap m;
   const uint64_t Eb = static_cast<uint64_t>(a.elems_per_chunk) * ES;
-  const uint64_t SLb = static_cast<uint64_t>(a.slice_elems) * ES;
-  const uint64_t jo = static_cast<uint64_t>(j) * SLb;
-  m.seg = a.seg_bytes;
+  const uint32_t nunits = static_cast<uint32_t>((Eb + kUnit - 1) / kUnit);  // Eb < 2^31
+  const uint64_t lo = static_cast<uint64_t>(j * nunits / a.nchannels) * kUnit;
+  const uint64_t hi = min(static_cast<uint64_t>((j + 1) * nunits / a.nchannels) * kUnit, Eb);
+  m.seg = seg;
   m.chunk_stride = Eb * a.ntrees;
-  m.first = static_cast<uint64_t>(t) * Eb + jo;
-  m.sl_full = static_cast<uint32_t>(jo < Eb ? min(SLb, Eb - jo) : 0);
+  m.first = static_cast<uint64_t>(t) * Eb + lo;
+  m.sl_full = static_cast<uint32_t>(hi > lo ? hi - lo : 0);
   m.nseg = (m.sl_full + m.seg - 1) / m.seg;
   const uint32_t K = a.K[t];
   const uint64_t nbytes = a.count * ES;
@@ -316,8 +323,8 @@ __device__ __forceinline__ SegMap seg_map(const LaunchArgs &a, int t, int j) {
   m.nseg_last = 0;
   if (K > 0 && (C % a.ntrees) == static_cast<uint64_t>(t) && nbytes < (C + 1) * Eb) {
     m.kfull = K - 1;  // this tree carries the short last chunk
-    const uint64_t s0 = C * Eb + jo;
-    m.last_len = static_cast<uint32_t>(s0 < nbytes ? min(SLb, nbytes - s0) : 0);
+    const uint64_t s0 = C * Eb + lo;
+    m.last_len = static_cast<uint32_t>(s0 < nbytes ? min(static_cast<uint64_t>(m.sl_full), nbytes - s0) : 0);
     const uint32_t aligned = m.last_len & ~15u;
     m.nseg_last = (aligned + m.seg - 1) / m.seg + ((m.last_len & 15u) ? 1 : 0);
   }
@@ -452,7 +459,7 @@ __device__ void control_warp_tma(const LaunchArgs &a, const TreeParams &p, int r
   const uint64_t base = a.base[t];
   const int stride = j * kFlagStrideU64;
   const Endpoints e = endpoints(a, p, role);
-  const SegMap m = seg_map<ES>(a, t, j);
+  const SegMap m = seg_map<ES>(a, t, j, a.seg_bytes);
   // upstream counters: UP waits on each child's head, DOWN on my own semaphore
   const uint64_t *up = nullptr;
   if (role == kRoleUp) {
@@ -598,7 +605,7 @@ __device__ void data_warp_tma(const LaunchArgs &a, const TreeParams &p, int role
   constexpr int ES = DT == kBFloat16 ? 2 : 4;
   const int lane = threadIdx.x & 31;
   const Endpoints e = endpoints(a, p, role);
-  const SegMap m = seg_map<ES>(a, t, j);
+  const SegMap m = seg_map<ES>(a, t, j, a.seg_bytes);
   for (uint32_t G = 0; G < m.total; ++G) {
     const int st = G % kStages;
     if (!mbar_wait(&sh.full[st], (G / kStages) & 1, &sh.abort)) return;
@@ -682,159 +689,101 @@ __device__ void control_warp_lsu(const LaunchArgs &a, const TreeParams &p, int r
   leaf_wait<SYS>(a, p, role, t, j);
 }
 
-// Item geometry of one (tree, channel) stream in 16-byte vectors.
-struct VecMap {
-  uint64_t first;         // byte offset of slice j of tree-local chunk 0
-  uint64_t chunk_stride;  // bytes between consecutive tree-local chunks
-  uint32_t nv_full;       // vectors of a full slice
-  uint32_t nv_last;       // vectors of the short last chunk's slice (if this tree has it)
-  uint32_t kfull;         // chunks with a full slice (K or K-1)
-  uint32_t ragged;        // bytes after the last whole vector of the buffer (0..15)
-};
-
-template <int ES>
-__device__ __forceinline__ VecMap vec_map(const LaunchArgs &a, int t, int j) {
-  const SegMap s = seg_map<ES>(a, t, j);
-  VecMap m;
-  m.first = s.first;
-  m.chunk_stride = s.chunk_stride;
-  m.nv_full = s.sl_full / 16;
-  m.kfull = s.kfull;
-  m.nv_last = s.last_len / 16;
-  m.ragged = s.last_len & 15u;
-  return m;
-}
-
-// Normalise (k, v) so that v < vectors(k), or k == K (past the end).
-__device__ __forceinline__ void vec_norm(const VecMap &m, uint32_t K, uint32_t &k, uint32_t &v) {
-  while (k < K) {
-    const uint32_t n = k < m.kfull ? m.nv_full : m.nv_last;
-    if (v < n) return;
-    v -= n;
-    ++k;
-  }
-}
-
+// One data warp's stream: blocks G = w, w+W, ... of 32*U vectors (512*U bytes).
+// A block lies inside one chunk's slice, so the readiness check and the base
+// address are warp-uniform; lane l handles vectors l + 32u, u < U.
 template <int DT, int NIN, int NOUT, int U>
-__device__ void lsu_stream(const LaunchArgs &a, const Endpoints &e, const VecMap &m, uint32_t K,
-                           int w, int W, Shared &sh, bool do_ragged) {
+__device__ void lsu_stream(const LaunchArgs &a, const Endpoints &e, int t, int j, int w, int W,
+                           Shared &sh) {
+  constexpr int ES = DT == kBFloat16 ? 2 : 4;
   const int lane = threadIdx.x & 31;
-  const uint32_t step = static_cast<uint32_t>(W) * 32;
-  uint32_t k = 0, v = static_cast<uint32_t>(w) * 32 + lane;
-  vec_norm(m, K, k, v);
+  const uint32_t K = a.K[t];
+  const SegMap m = seg_map<ES>(a, t, j, 512u * U);
   uint64_t ready = 0;
   uint32_t done_reported = 0;
-  bool ragged_left = do_ragged;
-  while (true) {
-    const uint32_t k0 = __shfl_sync(0xffffffffu, k, 0);
-    if (k0 >= K) break;
-    // every lane's next item must be in a ready chunk before a round can start
-    const uint32_t kneed = __reduce_max_sync(0xffffffffu, k < K ? k : 0);
-    if (kneed >= ready) {
+  for (uint32_t G = w; G < m.total; G += W) {
+    const uint32_t k = seg_chunk(m, G);
+    if (k >= ready) {
       uint64_t r = 0;
       if (lane == 0) {
         do {
           r = ld_acquire_cta(&sh.ready);
-        } while (r <= kneed && !*reinterpret_cast<volatile int *>(&sh.abort));
+        } while (r <= k && !*reinterpret_cast<volatile int *>(&sh.abort));
       }
       r = __shfl_sync(0xffffffffu, r, 0);
-      if (r <= kneed) return;  // aborted
+      if (r <= k) return;  // aborted
       ready = r;
     }
-    uint32_t kk[U], vv[U];
-    uint32_t ck = k, cv = v;
-    int rounds = 0;
+    uint64_t off;
+    uint32_t len;
+    seg_range(m, G, &off, &len);
+    if (len >= 16) {
+      const uint32_t nvec = len / 16;
+      const char *s0 = e.src[0] + off + lane * 16;
+      uint4 x[U][NIN];
 #pragma unroll
-    for (int u = 0; u < U; ++u) {
-      kk[u] = ck;
-      vv[u] = cv;
-      const uint32_t kmax = __reduce_max_sync(0xffffffffu, ck < K ? ck : 0);
-      const bool any = __any_sync(0xffffffffu, ck < K);
-      if (rounds == u && any && kmax < ready) {
-        rounds = u + 1;
-        cv += step;
-        vec_norm(m, K, ck, cv);
+      for (int u = 0; u < U; ++u) {
+        if (lane + 32u * u < nvec) {
+#pragma unroll
+          for (int q = 0; q < NIN; ++q)
+            x[u][q] = __ldcg(reinterpret_cast<const uint4 *>(e.src[q] + off + lane * 16 + 512u * u));
+        }
       }
-    }
-    uint4 x[U][NIN];
+      (void)s0;
 #pragma unroll
-    for (int u = 0; u < U; ++u) {
-      if (u < rounds && kk[u] < K) {
-        const uint64_t off = m.first + kk[u] * m.chunk_stride + static_cast<uint64_t>(vv[u]) * 16;
+      for (int u = 0; u < U; ++u) {
+        if (lane + 32u * u < nvec) {
+          const uint4 r = Combine<DT>::template vec<NIN>(x[u]);
 #pragma unroll
-        for (int q = 0; q < NIN; ++q) x[u][q] = __ldcg(reinterpret_cast<const uint4 *>(e.src[q] + off));
+          for (int q = 0; q < NOUT; ++q)
+            *reinterpret_cast<uint4 *>(e.dst[q] + off + lane * 16 + 512u * u) = r;
+        }
       }
+    } else {
+      combine_scalar<DT>(e.src, NIN, e.dst, NOUT, off, len);  // ragged end of the buffer
     }
-#pragma unroll
-    for (int u = 0; u < U; ++u) {
-      if (u < rounds && kk[u] < K) {
-        const uint64_t off = m.first + kk[u] * m.chunk_stride + static_cast<uint64_t>(vv[u]) * 16;
-        const uint4 r = Combine<DT>::template vec<NIN>(x[u]);
-#pragma unroll
-        for (int q = 0; q < NOUT; ++q) *reinterpret_cast<uint4 *>(e.dst[q] + off) = r;
-      }
-    }
-    k = ck;
-    v = cv;
-    uint32_t d = __shfl_sync(0xffffffffu, k, 0);  // lane 0 holds the warp's smallest item
-    if (ragged_left && d >= K) d = K - 1;
+    const uint32_t next = G + W;
+    const uint32_t d = next < m.total ? seg_chunk(m, next) : K;
     if (d > done_reported) {
-      __syncwarp();
+      __syncwarp();  // every lane's stores precede the release
       if (lane == 0) st_release_cta(&sh.done[w], d);
       done_reported = d;
     }
   }
-  if (ragged_left) {  // sub-vector tail at the end of the buffer (in the last chunk)
-    if (ready < K) {
-      uint64_t r = 0;
-      if (lane == 0) {
-        do {
-          r = ld_acquire_cta(&sh.ready);
-        } while (r < K && !*reinterpret_cast<volatile int *>(&sh.abort));
-      }
-      r = __shfl_sync(0xffffffffu, r, 0);
-      if (r < K) return;  // aborted
-    }
-    const uint64_t off = m.first + static_cast<uint64_t>(m.kfull) * m.chunk_stride +
-                         static_cast<uint64_t>(m.nv_last) * 16;
-    combine_scalar<DT>(e.src, NIN, e.dst, NOUT, off, m.ragged);
+  if (done_reported < K) {
+    __syncwarp();
+    if (lane == 0) st_release_cta(&sh.done[w], K);
   }
-  __syncwarp();
-  if (lane == 0) st_release_cta(&sh.done[w], K);
 }
 
 template <int DT, int NIN>
-__device__ __forceinline__ void lsu_nout(const LaunchArgs &a, const Endpoints &e, const VecMap &m,
-                                         uint32_t K, int w, int W, Shared &sh, bool rag) {
-  constexpr int U = NIN == 1 ? 8 : (NIN == 2 ? 6 : 4);
+__device__ __forceinline__ void lsu_nout(const LaunchArgs &a, const Endpoints &e, int t, int j,
+                                         int w, int W, Shared &sh) {
+  constexpr int U = NIN == 1 ? 8 : 4;  // block = 4 KB (copies) or 2 KB (combines)
   switch (e.nout) {
-    case 1: lsu_stream<DT, NIN, 1, U>(a, e, m, K, w, W, sh, rag); break;
-    case 2: lsu_stream<DT, NIN, 2, U>(a, e, m, K, w, W, sh, rag); break;
-    default: lsu_stream<DT, NIN, 3, U>(a, e, m, K, w, W, sh, rag); break;
+    case 1: lsu_stream<DT, NIN, 1, U>(a, e, t, j, w, W, sh); break;
+    case 2: lsu_stream<DT, NIN, 2, U>(a, e, t, j, w, W, sh); break;
+    default: lsu_stream<DT, NIN, 3, U>(a, e, t, j, w, W, sh); break;
   }
 }
 
 template <int DT>
 __device__ void data_warp_lsu(const LaunchArgs &a, const TreeParams &p, int role, int t, int j,
                               int w, int W, Shared &sh) {
-  constexpr int ES = DT == kBFloat16 ? 2 : 4;
   const Endpoints e = endpoints(a, p, role);
-  const VecMap m = vec_map<ES>(a, t, j);
-  const uint32_t K = a.K[t];
-  const bool rag = w == 0 && m.ragged != 0;
   if (e.nout == 0) {  // nothing to write (cannot happen for scheduled tasks)
-    if ((threadIdx.x & 31) == 0) st_release_cta(&sh.done[w], K);
+    if ((threadIdx.x & 31) == 0) st_release_cta(&sh.done[w], a.K[t]);
     return;
   }
   switch (e.nin) {
-    case 1: lsu_nout<DT, 1>(a, e, m, K, w, W, sh, rag); break;
-    case 2: lsu_nout<DT, 2>(a, e, m, K, w, W, sh, rag); break;
-    default: lsu_nout<DT, 3>(a, e, m, K, w, W, sh, rag); break;
+    case 1: lsu_nout<DT, 1>(a, e, t, j, w, W, sh); break;
+    case 2: lsu_nout<DT, 2>(a, e, t, j, w, W, sh); break;
+    default: lsu_nout<DT, 3>(a, e, t, j, w, W, sh); break;
   }
 }
 
 template <int DT, bool SYS>
-__global__ void __launch_bounds__(kMaxThreads) tree_allreduce_kernel(const LaunchArgs a) {
+__global__ void __launch_bounds__(kMaxThreads, kMinBlocksPerSm) tree_allreduce_kernel(const LaunchArgs a) {
   __shared__ Shared sh;
   extern __shared__ __align__(128) char stages[];
   const Task task = a.tasks[blockIdx.x];
