@@ -69,7 +69,7 @@ struct TreeParams {
 };
 
 enum Role { kRoleUp = 0, kRoleDown = 1 };
-enum Datapath { kDatapathLsu = 0, kDatapathTma = 1 };
+enum Datapath { kDatapathLsu = 0, kDatapathTma = 1, kDatapathAsync = 2 };
 
 enum { kAllChannels = -1 };  // a pulled leaf's single task covers every channel
 
@@ -85,13 +85,13 @@ struct LaunchArgs {
   const TreeParams *params;   // [local_rank * ntrees + tree]
   uint64_t count;             // elements
   uint32_t elems_per_chunk;   // E
-  uint32_t pad_slice;         // (unused) channel slices are derived in-kernel, see seg_map
+  uint32_t pad0;
   uint32_t ntrees;
   uint32_t nchannels;
   uint32_t K[kMaxTrees];      // tree-local chunk counts
   uint64_t base[kMaxTrees];   // counter base of this call per tree
   int overlap;                // 1 = C1, 0 = B
-  int datapath;               // kDatapathLsu (register-staged) or kDatapathTma
+  int datapath;               // kDatapathLsu (register-staged), kDatapathTma, kDatapathAsync (cp.async rings)
   uint64_t timeout_ns;        // watchdog
   int *err;                   // mapped host word; nonzero = abort
   uint64_t *trace;            // optional landing trace

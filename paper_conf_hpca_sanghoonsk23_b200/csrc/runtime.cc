@@ -489,7 +489,7 @@ ccube_result_t allreduce_impl(void *const *bufs, size_t count, ccube_dtype_t dty
 
   // all CTAs spin on each other: they must be co-resident
   const int cta_threads = g.threads + 32;  // data warps + the control warp
-  auto key = std::make_pair((int)dtype * 2 + g.datapath,
+  auto key = std::make_pair((int)dtype * 4 + g.datapath,
                             cta_threads * 1024 + (int)(g.seg_bytes >> 4));
   if (!g.max_blocks.count(key)) {
     int b = 0;
@@ -681,7 +681,12 @@ ccube_result_t ccube_init(const ccube_world_t *world, ccube_tree_kind_t tree_kin
   g.channels = channels;
   g.threads = threads;
   g.transport = transport;
-  g.datapath = env_int("CCUBE_DATAPATH_TMA", 0) ? kDatapathTma : kDatapathLsu;
+  g.datapath = env_int("CCUBE_DATAPATH", kDatapathAsync);
+  if (env_int("CCUBE_DATAPATH_TMA", 0)) g.datapath = kDatapathTma;
+  if (g.datapath < kDatapathLsu || g.datapath > kDatapathAsync) {
+    g = Comm();
+    return fail(CCUBE_ERR_INVALID_ARG, "CCUBE_DATAPATH must be 0 (lsu), 1 (tma) or 2 (async)");
+  }
   g.seg_bytes = static_cast<uint32_t>(env_int("CCUBE_SEG_BYTES", 16384));
   if (g.seg_bytes < 1024 || g.seg_bytes > 16384 || g.seg_bytes % 1024) {
     g = Comm();

@@ -361,6 +361,55 @@ __device__ __forceinline__ void seg_range(const SegMap &m, uint32_t G, uint64_t 
   }
 }
 
+// Incremental form of seg_chunk/seg_range for a warp that takes every W-th block.
+struct BlockIter {
+  uint32_t G;    // block index
+  uint32_t k;    // its chunk (tree-local)
+  uint32_t s;    // its segment inside the chunk slice
+  uint64_t off;  // byte offset in the buffer
+  uint32_t len;  // bytes (< 16: ragged buffer end)
+};
+
+__device__ __forceinline__ void block_fill(const SegMap &m, BlockIter &it) {
+  if (it.G >= m.total) return;
+  const uint64_t base = m.first + static_cast<uint64_t>(it.k) * m.chunk_stride;
+  if (it.k < m.kfull) {
+    it.off = base + static_cast<uint64_t>(it.s) * m.seg;
+    it.len = min(m.seg, m.sl_full - it.s * m.seg);
+    return;
+  }
+  const uint32_t aligned = m.last_len & ~15u;
+  const uint32_t full_segs = (aligned + m.seg - 1) / m.seg;
+  if (it.s < full_segs) {
+    it.off = base + static_cast<uint64_t>(it.s) * m.seg;
+    it.len = min(m.seg, aligned - it.s * m.seg);
+  } else {
+    it.off = base + aligned;
+    it.len = m.last_len - aligned;
+  }
+}
+
+__device__ __forceinline__ BlockIter block_iter(const SegMap &m, uint32_t G) {
+  BlockIter it;
+  it.G = G;
+  it.k = seg_chunk(m, G);
+  it.s = G - it.k * m.nseg;
+  it.off = 0;
+  it.len = 0;
+  block_fill(m, it);
+  return it;
+}
+
+__device__ __forceinline__ void block_next(const SegMap &m, BlockIter &it, uint32_t W) {
+  it.G += W;
+  it.s += W;
+  while (it.k < m.kfull && it.s >= m.nseg) {  // full chunks: nseg segments each
+    it.s -= m.nseg;
+    ++it.k;
+  }
+  block_fill(m, it);
+}
+
 // Sources and destinations of a task (a4/a5/a6).
 struct Endpoints {
   const char *src[kMaxIn];
@@ -701,8 +750,12 @@ __device__ void lsu_stream(const LaunchArgs &a, const Endpoints &e, int t, int j
   const SegMap m = seg_map<ES>(a, t, j, 512u * U);
   uint64_t ready = 0;
   uint32_t done_reported = 0;
-  for (uint32_t G = w; G < m.total; G += W) {
-    const uint32_t k = seg_chunk(m, G);
+  // Block iterator: this warp's blocks G = w, w+W, ... as (chunk k, segment s),
+  // advanced without divisions so the next addresses are ready as soon as the
+  // current loads are issued (the loop is load-latency bound).
+  BlockIter it = block_iter(m, w);
+  while (it.k < K && it.G < m.total) {
+    const uint32_t k = it.k;
     if (k >= ready) {
       uint64_t r = 0;
       if (lane == 0) {
@@ -714,12 +767,10 @@ __device__ void lsu_stream(const LaunchArgs &a, const Endpoints &e, int t, int j
       if (r <= k) return;  // aborted
       ready = r;
     }
-    uint64_t off;
-    uint32_t len;
-    seg_range(m, G, &off, &len);
+    const uint64_t off = it.off;
+    const uint32_t len = it.len;
     if (len >= 16) {
       const uint32_t nvec = len / 16;
-      const char *s0 = e.src[0] + off + lane * 16;
       uint4 x[U][NIN];
 #pragma unroll
       for (int u = 0; u < U; ++u) {
@@ -729,7 +780,7 @@ __device__ void lsu_stream(const LaunchArgs &a, const Endpoints &e, int t, int j
             x[u][q] = __ldcg(reinterpret_cast<const uint4 *>(e.src[q] + off + lane * 16 + 512u * u));
         }
       }
-      (void)s0;
+      block_next(m, it, W);  // overlaps the loads
 #pragma unroll
       for (int u = 0; u < U; ++u) {
         if (lane + 32u * u < nvec) {
@@ -741,9 +792,9 @@ __device__ void lsu_stream(const LaunchArgs &a, const Endpoints &e, int t, int j
       }
     } else {
       combine_scalar<DT>(e.src, NIN, e.dst, NOUT, off, len);  // ragged end of the buffer
+      block_next(m, it, W);
     }
-    const uint32_t next = G + W;
-    const uint32_t d = next < m.total ? seg_chunk(m, next) : K;
+    const uint32_t d = it.G < m.total ? it.k : K;
     if (d > done_reported) {
       __syncwarp();  // every lane's stores precede the release
       if (lane == 0) st_release_cta(&sh.done[w], d);
@@ -782,6 +833,156 @@ __device__ void data_warp_lsu(const LaunchArgs &a, const TreeParams &p, int role
   }
 }
 
+// ---- ASYNC path (default): per-lane cp.async rings ------------------------------
+// Same work split as the LSU path (warp w takes blocks G = w, w+W, ... of 32*kAU
+// vectors), but every lane stages ITS OWN 16-byte vectors of up to kRing/NIN
+// blocks ahead through shared memory with cp.async (LDGSTS): loads stay in flight
+// without holding registers, so each warp keeps ~12 KB of reads outstanding
+// continuously instead of one register round at a time.  A lane only ever reads
+// back what it copied itself, so cp.async.wait_group alone orders the data (no
+// barrier, no cross-proxy fence).  Readiness is checked per block before its loads
+// are issued, exactly as in the LSU path.
+constexpr int kAU = 2;                       // vectors per lane per source per block
+constexpr uint32_t kABlock = 512u * kAU;     // bytes per source per block (1 KB)
+constexpr int kRing = 12;                    // source-blocks in flight per warp
+constexpr uint32_t kRingBytes = kRing * kABlock;  // shared memory per data warp
+
+__device__ __forceinline__ void cp_async16(uint32_t smem, const void *gmem) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem), "l"(gmem) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() {
+  asm volatile("cp.async.commit_group;" ::: "memory");
+}
+template <int N>
+__device__ __forceinline__ void cp_async_wait() {
+  asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
+}
+// wait until at most `pending` (0 <= pending < S) groups are outstanding
+template <int S>
+__device__ __forceinline__ void cp_async_wait_dyn(uint32_t pending) {
+  if constexpr (S > 1) {
+    if (pending >= S - 1) {
+      cp_async_wait<S - 1>();
+      return;
+    }
+    cp_async_wait_dyn<S - 1>(pending);
+  } else {
+    cp_async_wait<0>();
+  }
+}
+
+template <int DT, int NIN, int NOUT>
+__device__ void async_stream(const LaunchArgs &a, const Endpoints &e, int t, int j, int w, int W,
+                             Shared &sh, char *ring) {
+  constexpr int ES = DT == kBFloat16 ? 2 : 4;
+  constexpr int S = kRing / NIN;  // blocks in flight
+  const int lane = threadIdx.x & 31;
+  const uint32_t K = a.K[t];
+  const SegMap m = seg_map<ES>(a, t, j, kABlock);
+  const uint32_t nb = m.total > static_cast<uint32_t>(w) ? (m.total - w + W - 1) / W : 0;
+  const uint32_t my = smem_u32(ring) + lane * 16;
+  uint64_t ready = 0;
+  uint32_t issued = 0, done_reported = 0;
+  for (uint32_t i = 0; i < nb; ++i) {
+    // top up: issue the loads of blocks i .. i+S-1 that are ready
+    while (issued < nb && issued < i + S) {
+      const uint32_t G = w + issued * W;
+      const uint32_t k = seg_chunk(m, G);
+      if (k >= ready) {
+        uint64_t r = 0;
+        if (lane == 0) {
+          r = ld_acquire_cta(&sh.ready);
+          if (issued == i)  // nothing in flight to work on: wait for it
+            while (r <= k && !*reinterpret_cast<volatile int *>(&sh.abort))
+              r = ld_acquire_cta(&sh.ready);
+        }
+        r = __shfl_sync(0xffffffffu, r, 0);
+        if (r > ready) ready = r;
+        if (k >= ready) {
+          if (issued == i) return;  // aborted
+          break;                    // work on what is in flight, re-check later
+        }
+      }
+      uint64_t off;
+      uint32_t len;
+      seg_range(m, G, &off, &len);
+      const uint32_t st = (issued % S) * NIN * kABlock;
+      if (len >= 16) {
+        const uint32_t nvec = len / 16;
+#pragma unroll
+        for (int u = 0; u < kAU; ++u)
+          if (lane + 32u * u < nvec) {
+#pragma unroll
+            for (int q = 0; q < NIN; ++q)
+              cp_async16(my + st + q * kABlock + 512u * u, e.src[q] + off + lane * 16 + 512u * u);
+          }
+      }
+      cp_async_commit();  // one group per block (empty for the ragged tail)
+      ++issued;
+    }
+    cp_async_wait_dyn<S>(issued - i - 1);
+    const uint32_t G = w + i * W;
+    uint64_t off;
+    uint32_t len;
+    seg_range(m, G, &off, &len);
+    if (len >= 16) {
+      const uint32_t nvec = len / 16;
+      const char *stage = ring + (i % S) * NIN * kABlock + lane * 16;
+#pragma unroll
+      for (int u = 0; u < kAU; ++u) {
+        if (lane + 32u * u < nvec) {
+          uint4 x[NIN];
+#pragma unroll
+          for (int q = 0; q < NIN; ++q)
+            x[q] = *reinterpret_cast<const uint4 *>(stage + q * kABlock + 512u * u);
+          const uint4 r = Combine<DT>::template vec<NIN>(x);
+#pragma unroll
+          for (int q = 0; q < NOUT; ++q)
+            *reinterpret_cast<uint4 *>(e.dst[q] + off + lane * 16 + 512u * u) = r;
+        }
+      }
+    } else {
+      combine_scalar<DT>(e.src, NIN, e.dst, NOUT, off, len);  // ragged end of the buffer
+    }
+    const uint32_t d = i + 1 < nb ? seg_chunk(m, G + W) : K;
+    if (d > done_reported) {
+      __syncwarp();  // every lane's stores precede the release
+      if (lane == 0) st_release_cta(&sh.done[w], d);
+      done_reported = d;
+    }
+  }
+  if (done_reported < K) {
+    __syncwarp();
+    if (lane == 0) st_release_cta(&sh.done[w], K);
+  }
+}
+
+template <int DT, int NIN>
+__device__ __forceinline__ void async_nout(const LaunchArgs &a, const Endpoints &e, int t, int j,
+                                           int w, int W, Shared &sh, char *ring) {
+  switch (e.nout) {
+    case 1: async_stream<DT, NIN, 1>(a, e, t, j, w, W, sh, ring); break;
+    case 2: async_stream<DT, NIN, 2>(a, e, t, j, w, W, sh, ring); break;
+    default: async_stream<DT, NIN, 3>(a, e, t, j, w, W, sh, ring); break;
+  }
+}
+
+template <int DT>
+__device__ void data_warp_async(const LaunchArgs &a, const TreeParams &p, int role, int t, int j,
+                                int w, int W, Shared &sh, char *stages) {
+  const Endpoints e = endpoints(a, p, role);
+  char *ring = stages + static_cast<size_t>(w) * kRingBytes;
+  if (e.nout == 0) {
+    if ((threadIdx.x & 31) == 0) st_release_cta(&sh.done[w], a.K[t]);
+    return;
+  }
+  switch (e.nin) {
+    case 1: async_nout<DT, 1>(a, e, t, j, w, W, sh, ring); break;
+    case 2: async_nout<DT, 2>(a, e, t, j, w, W, sh, ring); break;
+    default: async_nout<DT, 3>(a, e, t, j, w, W, sh, ring); break;
+  }
+}
+
 template <int DT, bool SYS>
 __global__ void __launch_bounds__(kMaxThreads, kMinBlocksPerSm) tree_allreduce_kernel(const LaunchArgs a) {
   __shared__ Shared sh;
@@ -811,6 +1012,11 @@ __global__ void __launch_bounds__(kMaxThreads, kMinBlocksPerSm) tree_allreduce_k
       control_warp_tma<ES, SYS>(a, p, task.role, task.tree, task.channel, sh, stages);
     else
       data_warp_tma<DT>(a, p, task.role, task.tree, task.channel, warp - 1, W, sh, stages);
+  } else if (a.datapath == kDatapathAsync) {
+    if (warp == 0)
+      control_warp_lsu<SYS>(a, p, task.role, task.tree, task.channel, W, sh);
+    else
+      data_warp_async<DT>(a, p, task.role, task.tree, task.channel, warp - 1, W, sh, stages);
   } else {
     if (warp == 0)
       control_warp_lsu<SYS>(a, p, task.role, task.tree, task.channel, W, sh);
@@ -843,13 +1049,15 @@ __global__ void gate_kernel(const GateArgs g) {
   }
 }
 
-size_t stage_bytes(int datapath, uint32_t seg) {
-  return datapath == kDatapathTma ? static_cast<size_t>(kStages) * kMaxIn * seg : 0;
+size_t stage_bytes(int datapath, uint32_t seg, int threads) {
+  if (datapath == kDatapathTma) return static_cast<size_t>(kStages) * kMaxIn * seg;
+  if (datapath == kDatapathAsync) return static_cast<size_t>(threads / 32 - 1) * kRingBytes;
+  return 0;
 }
 
 template <int DT, bool SYS>
 int launch_t(const LaunchArgs &a, int grid, int threads, cudaStream_t s) {
-  const size_t smem = stage_bytes(a.datapath, a.seg_bytes);
+  const size_t smem = stage_bytes(a.datapath, a.seg_bytes, threads);
   cudaError_t e = cudaFuncSetAttribute(tree_allreduce_kernel<DT, SYS>,
                                        cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        static_cast<int>(smem));
@@ -920,7 +1128,7 @@ int query_max_blocks_per_sm(int dtype, bool sys_scope, int threads, int datapath
       fn = sys_scope ? kernel_ptr<kBFloat16, true>() : kernel_ptr<kBFloat16, false>();
       break;
   }
-  const size_t smem = stage_bytes(datapath, seg_bytes);
+  const size_t smem = stage_bytes(datapath, seg_bytes, threads);
   cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        static_cast<int>(smem));
   if (e != cudaSuccess) return static_cast<int>(e);
