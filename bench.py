@@ -53,6 +53,18 @@ def parse():
     p.add_argument("--no-clocks", action="store_true")
     p.add_argument("--cpu-sample-chunks", type=int, default=0,
                    help="chunks per step for the oracle (0 = auto)")
+    p.add_argument("--mode", choices=["allreduce", "iter"], default="allreduce",
+                   help="iter: only the chained-vs-unchained training iteration")
+    p.add_argument("--no-iter", action="store_true",
+                   help="skip the chained-iteration sub-benchmark in the default line")
+    p.add_argument("--iter-batch", type=int, default=64)
+    p.add_argument("--iter-steps", type=int, default=10)
+    p.add_argument("--iter-rounds", type=int, default=3)
+    p.add_argument("--iter-warmup", type=int, default=2)
+    p.add_argument("--iter-channels", type=int, default=4)
+    p.add_argument("--iter-tree", choices=["single", "double"], default="single")
+    p.add_argument("--iter-rank", type=int, default=1,
+                   help="loopback rank that hosts the model replica (1 = a leaf of tree 0)")
     a = p.parse_args()
     if a.dtype is None:
         a.dtype = "bfloat16" if a.workload == "vgg16" else "float32"
@@ -229,7 +241,6 @@ def run_ccube(a):
     if a.threads:
         ccube.set_threads(a.threads)
     ccube.set_overlap(bool(a.overlap))
-    info = ccube.get_info()
     stream = torch.cuda.Stream()
 
     def step():
@@ -342,25 +353,155 @@ def run_ccube(a):
                "sample": f"oracle.allreduce.replay on the first {nch} chunks ({sb} B per rank) "
                          f"of the {a.workload} gradient set, P={P}, {a.tree} tree; {dt:.2f} s"}
 
+    info = ccube.get_info()
+    ccube.finalize()
+    iteration = None
+    if not multi and not a.no_iter:
+        del bufs, pristine
+        torch.cuda.empty_cache()
+        try:
+            iteration = run_iteration(a, P, log=_log)
+        except Exception as e:  # noqa: BLE001 — reported in the line, the busbw stands
+            iteration = {"error": repr(e)}
+
     if rank == 0:
         line = {
             "metric": METRIC, "value": bw, "unit": "GB/s", "n_gpus": world,
             "steps": a.steps, "warmup": a.warmup, "ms_per_step": ms_step,
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
             "dtype": _dt(a.dtype), "data": "synthetic",
-            "config": dict(_config(a, P, nbytes), channels=info["channels"],
-                           threads=info["threads"],
+            "config": dict(_config(a, P, nbytes), channels=info["last_channels"],
+                           ctas=info["last_ctas"], threads=info["threads"],
                            l2="inputs (P x bytes_per_rank) larger than L2 and restored from a "
                               "pristine copy between timed steps (flushes L2)"),
             "algbw": alg, "busbw_frac_of_900": bw / NVLINK_NOMINAL_GBS,
             "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "clocks": clk,
             "gpu_launches": a.steps, "ranks_identical": ok,
             "ms_per_step_p10_p50_p90": [float(np.percentile(ms, q)) for q in (10, 50, 90)],
+            "iteration": iteration,
         }
         print(json.dumps(line), flush=True)
-    ccube.finalize()
     if multi:
         dist.destroy_process_group()
+
+
+# ------------------------------------------------------- chained training iteration
+ITER_MODES = ("compute", "B", "C1", "C2", "CC")   # paper's B / C1 / C2 / CC
+
+
+def run_iteration(a, P, log=None):
+    """Gradient-queue chaining (BASELINE.json configs[3]): synthetic ResNet-50
+    data-parallel iterations, loopback (P logical ranks on one GPU, one model
+    replica on local rank ``a.iter_rank``; the other ranks' backward output is
+    emulated by a copy of the replica's gradients, inside the compute phase).
+
+    Modes: compute (no AllReduce), B (non-overlapped tree, unchained), C1
+    (overlapped tree, unchained), C2 (B + per-layer gates), CC (C1 + gates).
+    Unchained: the next forward waits for the whole AllReduce.  Chained: each
+    layer's update+forward waits on its own gate (ccube_gradq_wait).
+    Returns {mode: ms per iteration} and exposed = T_mode - T_compute."""
+    import torch
+    import torch.nn.functional as F
+    import torchvision
+    from paper_conf_hpca_sanghoonsk23_b200 import ccube
+    from paper_conf_hpca_sanghoonsk23_b200.gradient_queue import attach_gradient_queue
+
+    dev = torch.device("cuda", torch.cuda.current_device())
+    torch.manual_seed(0)
+    torch.backends.cudnn.benchmark = True
+    model = torchvision.models.resnet50(weights=None).to(dev).to(memory_format=torch.channels_last)
+    rr = a.iter_rank % P
+    gq = attach_gradient_queue(model, lr=1e-3, world_size=P, local_rank=rr)
+    gq.update = True
+    B = a.iter_batch
+    x = torch.randn(B, 3, 224, 224, device=dev).to(memory_format=torch.channels_last)
+    y = torch.randint(0, 1000, (B,), device=dev)
+    others = [torch.zeros_like(gq.flat) for _ in range(P - 1)]
+    bufs = others[:rr] + [gq.flat] + others[rr:]
+    comp, comm = torch.cuda.Stream(), torch.cuda.Stream()
+    ccube.init_loopback(P, a.iter_tree, a.chunk_bytes)
+    res = {}
+    try:
+        ccube.set_channels(a.iter_channels)
+        gq.set_layers()
+
+        ev = lambda: torch.cuda.Event(enable_timing=True)  # noqa: E731
+
+        def one(mode, marks=None):
+            with torch.cuda.stream(comp):
+                with torch.autocast("cuda", dtype=torch.bfloat16):
+                    out = model(x)
+                    loss = F.cross_entropy(out.float(), y)
+                if marks is not None:
+                    marks["fwd_end"] = ev()
+                    marks["fwd_end"].record(comp)
+                comp.wait_stream(comm)    # the AllReduce is done reading/writing the queue
+                gq.zero_()
+                loss.backward()
+                for o in others:          # emulated replicas' backward output
+                    o.copy_(gq.flat)
+            if mode != "compute":
+                comm.wait_stream(comp)
+                if marks is not None:
+                    marks["ar0"] = ev()
+                    marks["ar0"].record(comm)
+                ccube.allreduce_tree_local(bufs, stream=comm)
+                if marks is not None:
+                    marks["ar1"] = ev()
+                    marks["ar1"].record(comm)
+                if mode in ("B", "C1"):
+                    comp.wait_stream(comm)
+
+        runs = {m: [] for m in ITER_MODES}
+        timeline = {}
+        for rnd in range(a.iter_rounds):          # modes interleaved, median over rounds
+            for mode in ITER_MODES:
+                ccube.set_overlap(mode in ("C1", "CC"))
+                gq.chained = mode in ("C2", "CC")
+                for _ in range(a.iter_warmup):
+                    one(mode)
+                torch.cuda.synchronize()
+                e0, e1 = ev(), ev()
+                e0.record(comp)
+                for _ in range(a.iter_steps):
+                    one(mode)
+                comp.wait_stream(comm)
+                e1.record(comp)
+                if rnd == 0:   # one instrumented pair: AllReduce of i, forward of i+1
+                    m0, m1 = {}, {}
+                    one(mode, m0)
+                    one(mode, m1)
+                    comp.wait_stream(comm)
+                torch.cuda.synchronize()
+                runs[mode].append(e0.elapsed_time(e1) / a.iter_steps)
+                if rnd == 0:
+                    tl = {"forward_end_after_allreduce_end_ms": None}
+                    if mode != "compute":
+                        tl["allreduce_ms"] = m0["ar0"].elapsed_time(m0["ar1"])
+                        tl["forward_end_after_allreduce_end_ms"] = \
+                            m0["ar1"].elapsed_time(m1["fwd_end"])
+                    timeline[mode] = tl
+                gq.chained = False
+                if log:
+                    log(f"[iter] round {rnd} {mode}: {runs[mode][-1]:.3f} ms/iter")
+        res = {m: float(np.median(v)) for m, v in runs.items()}
+    finally:
+        gq.remove()
+        ccube.finalize()
+    t0 = res["compute"]
+    out = {"unit": "ms/iter", "batch": B, "P": P, "tree": a.iter_tree,
+           "channels": a.iter_channels, "replica_rank": rr,
+           "model": "torchvision resnet50 (random init), bf16 autocast, channels_last",
+           "ms": res, "exposed_ms": {m: res[m] - t0 for m in ITER_MODES if m != "compute"},
+           "runs_ms": runs, "timeline": timeline, "rounds": a.iter_rounds,
+           "steps_per_round": a.iter_steps,
+           "note": "loopback: P logical ranks share one GPU's SMs and HBM with the compute"}
+    exp = out["exposed_ms"]
+    cut = lambda m, ref: (1 - exp[m] / exp[ref]) if exp[ref] > 0 else None  # noqa: E731
+    out["exposed_cut_CC_vs_B"] = cut("CC", "B")
+    out["exposed_cut_C2_vs_B"] = cut("C2", "B")      # chaining alone
+    out["exposed_cut_CC_vs_C1"] = cut("CC", "C1")    # chaining on top of the overlapped tree
+    return out
 
 
 def _port_loads(P, kind):
@@ -386,10 +527,31 @@ def _ncu_traffic():
         return None
 
 
+def _log(msg):
+    print(msg, file=sys.stderr, flush=True)
+
+
+def run_iter_only(a):
+    """--mode iter: only the chained-vs-unchained iteration (loopback, N=1)."""
+    import torch
+    torch.cuda.set_device(0)
+    it = run_iteration(a, a.ranks, log=_log)
+    line = {"metric": "iter time chained vs unchained (synthetic ResNet-50 DP iteration)",
+            "value": it["ms"]["CC"], "unit": "ms/iter", "n_gpus": 1,
+            "steps": a.iter_steps, "warmup": a.iter_warmup, "higher_is_better": False,
+            "dtype": "bf16 compute / f32 gradients", "data": "synthetic",
+            "config": {"workload": f"resnet50 iteration, batch {a.iter_batch}, P={a.ranks} "
+                                   f"logical ranks (loopback), {a.iter_tree} tree"},
+            "iteration": it}
+    print(json.dumps(line), flush=True)
+
+
 def main():
     a = parse()
     if a.impl == "reference":
         run_reference(a)
+    elif a.mode == "iter":
+        run_iter_only(a)
     else:
         run_ccube(a)
 

@@ -21,6 +21,9 @@
  *                         GPU; every rank's buffer is local HBM and one kernel
  *                         launch runs the same per-rank kernel body for all ranks.
  *                         Used for single-GPU parity tests and the 1-GPU bench.
+ *   Two processes on ONE GPU are refused (their spinning kernels only time-slice)
+ *   unless CCUBE_ALLOW_SHARED_GPU=1: the multi-process tests use that to run the
+ *   IPC / .sys-scope path on a single GPU.
  *
  * Conventions:
  *   - Collective calls (init, register, allreduce, finalize) must be made by all
@@ -178,11 +181,13 @@ CCUBE_API ccube_result_t ccube_finalize(void);
 
 CCUBE_API const char *ccube_last_error(void);
 
-/* Introspection (host-only, no CUDA needed). */
+/* Introspection (host-only, no CUDA needed).  channels/threads are the configured
+ * values (0 = auto); last_channels/last_ctas describe the most recent launch. */
 typedef struct {
   int initialized, world_size, rank, nlocal, ntrees, channels, threads, overlap, transport;
   size_t chunk_bytes;
   uint64_t epoch_base[2];
+  int last_channels, last_ctas;
 } ccube_info_t;
 CCUBE_API ccube_result_t ccube_get_info(ccube_info_t *info);
 

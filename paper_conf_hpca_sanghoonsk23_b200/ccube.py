@@ -63,7 +63,8 @@ class Info(ctypes.Structure):
     _fields_ = [("initialized", ctypes.c_int), ("world_size", ctypes.c_int),
                 ("rank", ctypes.c_int), ("nlocal", ctypes.c_int), ("ntrees", ctypes.c_int),
                 ("channels", ctypes.c_int), ("threads", ctypes.c_int), ("overlap", ctypes.c_int),
-                ("transport", ctypes.c_int), ("chunk_bytes", ctypes.c_size_t), ("epoch_base", ctypes.c_uint64 * 2)]
+                ("transport", ctypes.c_int), ("chunk_bytes", ctypes.c_size_t), ("epoch_base", ctypes.c_uint64 * 2),
+                ("last_channels", ctypes.c_int), ("last_ctas", ctypes.c_int)]
 
 
 _lib = None

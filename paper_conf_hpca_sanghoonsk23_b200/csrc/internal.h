@@ -66,10 +66,10 @@ struct TreeParams {
   int leaf_pull;                    // leaf on a PULL edge: publishes all chunks at once
   int self_local;                   // local index of this rank (trace)
   int child_local[kMaxChildren];    // local index of each child, -1 if remote (trace)
+  int child_interior[kMaxChildren]; // child has children: its buffer is re-read (DOWN)
 };
 
 enum Role { kRoleUp = 0, kRoleDown = 1 };
-enum Datapath { kDatapathLsu = 0, kDatapathTma = 1, kDatapathAsync = 2 };
 
 enum { kAllChannels = -1 };  // a pulled leaf's single task covers every channel
 
@@ -91,12 +91,11 @@ struct LaunchArgs {
   uint32_t K[kMaxTrees];      // tree-local chunk counts
   uint64_t base[kMaxTrees];   // counter base of this call per tree
   int overlap;                // 1 = C1, 0 = B
-  int datapath;               // kDatapathLsu (register-staged), kDatapathTma, kDatapathAsync (cp.async rings)
   uint64_t timeout_ns;        // watchdog
   int *err;                   // mapped host word; nonzero = abort
   uint64_t *trace;            // optional landing trace
   uint32_t trace_kmax;
-  uint32_t seg_bytes;         // TMA segment bytes per source (stage size)
+  int l2_hints;               // 1 = per-stream L2 eviction priorities (keep re-read data)
 };
 
 // Kernel launcher (tree_allreduce.cu).  Returns a cudaError_t as int.
@@ -105,7 +104,6 @@ int launch_tree_allreduce(const LaunchArgs &args, int dtype, bool sys_scope, int
 constexpr int kMaxGateCounters = 128;
 int launch_gate(const uint64_t *const *counters, const uint64_t *targets, int n, int *err,
                 uint64_t timeout_ns, bool sys_scope, void *stream);
-int query_max_blocks_per_sm(int dtype, bool sys_scope, int threads, int datapath,
-                            uint32_t seg_bytes, int *blocks);
+int query_max_blocks_per_sm(int dtype, bool sys_scope, int threads, int *blocks);
 
 }  // namespace ccube

@@ -162,6 +162,8 @@ struct Comm {
   uint32_t last_K[kMaxTrees] = {0, 0};
   uint64_t last_E = 0;
   int last_channels = 0;
+  int last_ctas = 0;
+  int l2_hints = 1;
   std::vector<size_t> layer_ends;
   std::vector<char *> flags_local;  // [nlocal]
   std::vector<char *> world_flags;  // [world]
@@ -170,8 +172,6 @@ struct Comm {
   std::vector<std::unique_ptr<Registration>> regs;
   std::map<std::pair<int, int>, TaskTable> tasks;  // (channels, overlap)
   int transport = CCUBE_TRANSPORT_AUTO;
-  uint32_t seg_bytes = 16384;  // TMA stage bytes per source
-  int datapath = kDatapathLsu;
   bool sys_scope = false;
   uint64_t timeout_ns = 10000ull * 1000000ull;
   int sm_count = 0;
@@ -328,6 +328,7 @@ ccube_result_t build_params(Registration *R) {
         p.child_buf[s] = R->world_buf[c];
         p.child_enq[s] = reinterpret_cast<uint64_t *>(g.world_flags[c] + flag_offset(t, kEnq, 0));
         p.child_local[s] = is_local(c) ? c - g.rank0 : -1;
+        p.child_interior[s] = tr.nchild[c] > 0;
         if (edge_is_pull(c, r)) {
           p.up_src[1 + s] = R->world_buf[c];
         } else {
@@ -489,12 +490,11 @@ ccube_result_t allreduce_impl(void *const *bufs, size_t count, ccube_dtype_t dty
 
   // all CTAs spin on each other: they must be co-resident
   const int cta_threads = g.threads + 32;  // data warps + the control warp
-  auto key = std::make_pair((int)dtype * 4 + g.datapath,
-                            cta_threads * 1024 + (int)(g.seg_bytes >> 4));
+  auto key = std::make_pair((int)dtype, cta_threads);
   if (!g.max_blocks.count(key)) {
     int b = 0;
     const int rc =
-        query_max_blocks_per_sm(dtype, g.sys_scope, cta_threads, g.datapath, g.seg_bytes, &b);
+        query_max_blocks_per_sm(dtype, g.sys_scope, cta_threads, &b);
     if (rc != cudaSuccess)
       return fail(CCUBE_ERR_CUDA, "occupancy query failed: %s",
                   cudaGetErrorString(static_cast<cudaError_t>(rc)));
@@ -525,8 +525,7 @@ ccube_result_t allreduce_impl(void *const *bufs, size_t count, ccube_dtype_t dty
   a.err = g.err_dev;
   a.trace = g.trace;
   a.trace_kmax = static_cast<uint32_t>(g.trace_kmax);
-  a.seg_bytes = g.seg_bytes;
-  a.datapath = g.datapath;
+  a.l2_hints = g.l2_hints;
   a.params = R->d_params;
 
   TaskTable *tt = nullptr;
@@ -544,6 +543,7 @@ ccube_result_t allreduce_impl(void *const *bufs, size_t count, ccube_dtype_t dty
   g.have_call = true;
   g.last_E = E;
   g.last_channels = J;
+  g.last_ctas = tt->n;
   for (int t = 0; t < g.ntrees; ++t) {
     g.last_base[t] = g.base[t];
     g.last_K[t] = a.K[t];
@@ -681,18 +681,8 @@ ccube_result_t ccube_init(const ccube_world_t *world, ccube_tree_kind_t tree_kin
   g.channels = channels;
   g.threads = threads;
   g.transport = transport;
-  g.datapath = env_int("CCUBE_DATAPATH", kDatapathAsync);
-  if (env_int("CCUBE_DATAPATH_TMA", 0)) g.datapath = kDatapathTma;
-  if (g.datapath < kDatapathLsu || g.datapath > kDatapathAsync) {
-    g = Comm();
-    return fail(CCUBE_ERR_INVALID_ARG, "CCUBE_DATAPATH must be 0 (lsu), 1 (tma) or 2 (async)");
-  }
-  g.seg_bytes = static_cast<uint32_t>(env_int("CCUBE_SEG_BYTES", 16384));
-  if (g.seg_bytes < 1024 || g.seg_bytes > 16384 || g.seg_bytes % 1024) {
-    g = Comm();
-    return fail(CCUBE_ERR_INVALID_ARG, "CCUBE_SEG_BYTES must be a multiple of 1024 in [1024, 16384]");
-  }
   g.overlap = 1;
+  g.l2_hints = env_int("CCUBE_L2_HINTS", 1);
   g.sys_scope = g.nproc > 1;
   g.timeout_ns = static_cast<uint64_t>(env_int("CCUBE_WATCHDOG_MS", 10000)) * 1000000ull;
   g.use_memop = env_int("CCUBE_GATE_KERNEL", 0) == 0;
@@ -716,6 +706,7 @@ ccube_result_t ccube_init(const ccube_world_t *world, ccube_tree_kind_t tree_kin
     g = Comm();
     return rc;
   }
+  const bool allow_shared = env_int("CCUBE_ALLOW_SHARED_GPU", 0) != 0;
   for (int p = 0; p < g.nproc; ++p) {
     const Hello &h = all[p];
     if (h.magic != mine.magic || h.world != P || h.nlocal != g.nlocal ||
@@ -727,13 +718,16 @@ ccube_result_t ccube_init(const ccube_world_t *world, ccube_tree_kind_t tree_kin
                   "tree %d chunk %llu)",
                   p, h.world, h.nlocal, h.rank, h.tree_kind, (unsigned long long)h.chunk_bytes);
     }
-    for (int q = 0; q < p; ++q)
+    // Several processes on one GPU only time-slice (no MPS): their spinning kernels
+    // make progress one context switch at a time.  Refused unless a test asks for it
+    // (CCUBE_ALLOW_SHARED_GPU=1 exercises the IPC / .sys-scope path on one GPU).
+    for (int q = 0; q < p && !allow_shared; ++q)
       if (strncmp(all[q].busid, h.busid, sizeof h.busid) == 0 &&
           strncmp(h.busid, "nodevice", 8) != 0) {
         g = Comm();
         return fail(CCUBE_ERR_UNSUPPORTED,
-                    "processes %d and %d share GPU %s: persistent spinning kernels of two "
-                    "processes cannot run concurrently on one GPU",
+                    "processes %d and %d share GPU %s: the spinning kernels of two processes "
+                    "only time-slice on one GPU (CCUBE_ALLOW_SHARED_GPU=1 permits it for tests)",
                     q, p, h.busid);
       }
   }
@@ -939,6 +933,8 @@ ccube_result_t ccube_get_info(ccube_info_t *info) {
   info->chunk_bytes = g.chunk_bytes;
   info->epoch_base[0] = g.base[0];
   info->epoch_base[1] = g.base[1];
+  info->last_channels = g.last_channels;
+  info->last_ctas = g.last_ctas;
   return CCUBE_SUCCESS;
 }
 

@@ -27,10 +27,6 @@ def main():
     p.add_argument("--chunks", default=str(256 << 10))
     p.add_argument("--iters", type=int, default=20)
     p.add_argument("--transport", default="auto")
-    p.add_argument("--seg", default="16384")
-    p.add_argument("--tma", default="2", help="datapath: 0 lsu, 1 tma, 2 async")
-    p.add_argument("--prefetch", default="0")
-    p.add_argument("--rel", default="4", help="CCUBE_RELEASE_EVERY values")
     p.add_argument("--bytes", type=int, default=0, help="override buffer bytes per rank")
     a = p.parse_args()
     tdt = {"float32": torch.float32, "bfloat16": torch.bfloat16, "int32": torch.int32}[a.dtype]
@@ -40,15 +36,10 @@ def main():
     bufs = [torch.randn(count, device="cuda").to(tdt) for _ in range(P)]
     flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
     s = torch.cuda.Stream()
-    for tree, ov, ch, th, cb, tp, sg, tma, pf, rel in itertools.product(
+    for tree, ov, ch, th, cb, tp in itertools.product(
             a.trees.split(","), a.overlap.split(","), a.channels.split(","), a.threads.split(","),
-            a.chunks.split(","), a.transport.split(","), a.seg.split(","), a.tma.split(","),
-            a.prefetch.split(","), a.rel.split(",")):
+            a.chunks.split(","), a.transport.split(",")):
         try:
-            os.environ["CCUBE_SEG_BYTES"] = sg
-            os.environ["CCUBE_DATAPATH"] = tma
-            os.environ["CCUBE_PREFETCH"] = pf
-            os.environ["CCUBE_RELEASE_EVERY"] = rel
             ccube.init_loopback(P, tree, int(cb))
             ccube.set_channels(int(ch))
             ccube.set_threads(int(th))
@@ -69,8 +60,9 @@ def main():
             nbytes = count * es
             busbw = nbytes / (med / 1e3) / 1e9 * 2 * (P - 1) / P
             hbm = 2 * P * nbytes / (med / 1e3) / 1e9
-            print(json.dumps({"tree": tree, "tma": int(tma), "prefetch": int(pf), "rel": int(rel), "transport": tp, "seg": int(sg), "overlap": int(ov),
-                              "channels": int(ch),
+            print(json.dumps({"P": P, "tree": tree, "transport": tp, "overlap": int(ov),
+                              "channels": ccube.get_info()["last_channels"],
+                              "ctas": ccube.get_info()["last_ctas"],
                               "threads": int(th), "chunk": int(cb), "ms": round(med, 4),
                               "busbw": round(busbw, 1), "hbm_algo_gbs": round(hbm, 1)}),
                   flush=True)
