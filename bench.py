@@ -41,7 +41,7 @@ def parse():
     p.add_argument("--impl", choices=["ccube", "reference"], default="ccube")
     p.add_argument("--workload", choices=["resnet50", "vgg16"], default="resnet50")
     p.add_argument("--dtype", choices=["float32", "bfloat16", "int32"], default=None)
-    p.add_argument("--tree", choices=["single", "double"], default=None)
+    p.add_argument("--tree", choices=["single", "double", "rotated"], default=None)
     p.add_argument("--ranks", type=int, default=8, help="logical ranks in loopback (N=1)")
     p.add_argument("--overlap", type=int, default=1, help="1 = C1, 0 = B")
     p.add_argument("--chunk-bytes", type=int, default=256 << 10)
@@ -58,11 +58,14 @@ def parse():
     p.add_argument("--no-iter", action="store_true",
                    help="skip the chained-iteration sub-benchmark in the default line")
     p.add_argument("--iter-batch", type=int, default=64)
+    p.add_argument("--iter-model", choices=["resnet50", "vgg16"], default="resnet50")
+    p.add_argument("--iter-fused-sgd", action="store_true",
+                   help="apply the SGD step inside the AllReduce kernel (f2)")
     p.add_argument("--iter-steps", type=int, default=10)
     p.add_argument("--iter-rounds", type=int, default=3)
     p.add_argument("--iter-warmup", type=int, default=2)
     p.add_argument("--iter-channels", type=int, default=4)
-    p.add_argument("--iter-tree", choices=["single", "double"], default="single")
+    p.add_argument("--iter-tree", choices=["single", "double", "rotated"], default="single")
     p.add_argument("--iter-rank", type=int, default=1,
                    help="loopback rank that hosts the model replica (1 = a leaf of tree 0)")
     a = p.parse_args()
@@ -409,21 +412,27 @@ def run_iteration(a, P, log=None):
     dev = torch.device("cuda", torch.cuda.current_device())
     torch.manual_seed(0)
     torch.backends.cudnn.benchmark = True
-    model = torchvision.models.resnet50(weights=None).to(dev).to(memory_format=torch.channels_last)
+    model = getattr(torchvision.models, a.iter_model)(weights=None)
+    model = model.to(dev).to(memory_format=torch.channels_last)
     rr = a.iter_rank % P
-    gq = attach_gradient_queue(model, lr=1e-3, world_size=P, local_rank=rr)
+    gq = attach_gradient_queue(model, lr=1e-3, world_size=P, local_rank=rr,
+                               fused_sgd=a.iter_fused_sgd)
     gq.update = True
     B = a.iter_batch
     x = torch.randn(B, 3, 224, 224, device=dev).to(memory_format=torch.channels_last)
     y = torch.randint(0, 1000, (B,), device=dev)
     others = [torch.zeros_like(gq.flat) for _ in range(P - 1)]
     bufs = others[:rr] + [gq.flat] + others[rr:]
+    wts = None
+    if a.iter_fused_sgd:   # the emulated replicas' weights, updated by the kernel too
+        ow = [gq.flat_w.clone() for _ in range(P - 1)]
+        wts = ow[:rr] + [gq.flat_w] + ow[rr:]
     comp, comm = torch.cuda.Stream(), torch.cuda.Stream()
     ccube.init_loopback(P, a.iter_tree, a.chunk_bytes)
     res = {}
     try:
         ccube.set_channels(a.iter_channels)
-        gq.set_layers()
+        gq.set_layers(weights=wts)
 
         ev = lambda: torch.cuda.Event(enable_timing=True)  # noqa: E731
 
@@ -458,6 +467,8 @@ def run_iteration(a, P, log=None):
             for mode in ITER_MODES:
                 ccube.set_overlap(mode in ("C1", "CC"))
                 gq.chained = mode in ("C2", "CC")
+                # compute-only has no AllReduce to ride on: the hooks update instead
+                gq.fused_sgd = a.iter_fused_sgd and mode != "compute"
                 for _ in range(a.iter_warmup):
                     one(mode)
                 torch.cuda.synchronize()
@@ -491,7 +502,9 @@ def run_iteration(a, P, log=None):
     t0 = res["compute"]
     out = {"unit": "ms/iter", "batch": B, "P": P, "tree": a.iter_tree,
            "channels": a.iter_channels, "replica_rank": rr,
-           "model": "torchvision resnet50 (random init), bf16 autocast, channels_last",
+           "fused_sgd": a.iter_fused_sgd,
+           "model": f"torchvision {a.iter_model} (random init), bf16 autocast, channels_last",
+           "grad_bytes_per_rank": gq.numel * 4,
            "ms": res, "exposed_ms": {m: res[m] - t0 for m in ITER_MODES if m != "compute"},
            "runs_ms": runs, "timeline": timeline, "rounds": a.iter_rounds,
            "steps_per_round": a.iter_steps,
@@ -507,7 +520,7 @@ def run_iteration(a, P, log=None):
 def _port_loads(P, kind):
     """Bytes each rank sends per direction per byte of buffer (library trees)."""
     from paper_conf_hpca_sanghoonsk23_b200 import ccube
-    ntrees = 2 if kind == "double" else 1
+    ntrees = {"single": 1, "double": 2, "rotated": P if P > 1 else 1}[kind]
     loads = [0.0] * P
     for t in range(ntrees):
         par = ccube.tree_parents(P, kind, t)
@@ -536,11 +549,11 @@ def run_iter_only(a):
     import torch
     torch.cuda.set_device(0)
     it = run_iteration(a, a.ranks, log=_log)
-    line = {"metric": "iter time chained vs unchained (synthetic ResNet-50 DP iteration)",
+    line = {"metric": f"iter time chained vs unchained (synthetic {a.iter_model} DP iteration)",
             "value": it["ms"]["CC"], "unit": "ms/iter", "n_gpus": 1,
             "steps": a.iter_steps, "warmup": a.iter_warmup, "higher_is_better": False,
             "dtype": "bf16 compute / f32 gradients", "data": "synthetic",
-            "config": {"workload": f"resnet50 iteration, batch {a.iter_batch}, P={a.ranks} "
+            "config": {"workload": f"{a.iter_model} iteration, batch {a.iter_batch}, P={a.ranks} "
                                    f"logical ranks (loopback), {a.iter_tree} tree"},
             "iteration": it}
     print(json.dumps(line), flush=True)

@@ -67,8 +67,17 @@ typedef enum {
 
 /* Tree kind.  SINGLE: one binary tree rooted at rank 0.  DOUBLE: two
  * complementary trees, the second "flipped to invert the nodes and leaves"
- * (fn4 P:L153); chunk c travels on tree c mod 2 (reading R4). */
-typedef enum { CCUBE_TREE_SINGLE = 0, CCUBE_TREE_DOUBLE = 1 } ccube_tree_kind_t;
+ * (fn4 P:L153); chunk c travels on tree c mod 2 (reading R4).
+ * ROTATED: the balanced multi-tree set (the NVSwitch form of the
+ * topology-aware trees of §IV): P trees, tree t = tree 0 with every
+ * rank v renamed (v + t) mod P, chunk c on tree c mod P.  Every rank plays every
+ * tree position once, so each GPU's NVLink port carries 2(P-1)/P of the buffer per
+ * direction — the bandwidth-optimal load, vs 2 for the double tree at P=8. */
+typedef enum {
+  CCUBE_TREE_SINGLE = 0,
+  CCUBE_TREE_DOUBLE = 1,
+  CCUBE_TREE_ROTATED = 2
+} ccube_tree_kind_t;
 
 /* Element type.  int32 adds wrap mod 2^32; fp32 adds are IEEE RN (no FMA, no FTZ);
  * bf16 is widened to fp32, added in the fixed order and rounded once (RNE) per
@@ -93,7 +102,7 @@ typedef struct {
 } ccube_world_t;
 
 #define CCUBE_MAX_RANKS 8
-#define CCUBE_MAX_CHANNELS 64
+#define CCUBE_MAX_CHANNELS 128
 #define CCUBE_DEFAULT_CHUNK_BYTES (256u * 1024u) /* 256 chunks for 64 MB */
 
 /* ccube_init — collective.  Builds the tree(s), allocates the
@@ -149,13 +158,30 @@ CCUBE_API ccube_result_t ccube_gradq_set_layers(const size_t *layer_end_elems, i
 CCUBE_API ccube_result_t ccube_gradq_wait(int layer_id, void *stream);
 CCUBE_API ccube_result_t ccube_gradq_wait_local(int local_rank, int layer_id, void *stream);
 
+/* ccube_gradq_set_sgd — fused SGD update at dequeue (the paper gates
+ * "update and forward" of layer l on its chunks).  When set, every
+ * allreduce also applies, on every rank, w[e] <- w[e] - alpha * g[e] to that rank's
+ * fp32 weights, where g is the reduced (summed) gradient — alpha = lr / P gives the
+ * averaged SGD step (R14) — as two IEEE-rounded operations, no FMA (reading R18).
+ * The step is done by the task that already handles the rank's final gradient (the
+ * root's reduce, an interior rank's broadcast, an extra pass at each leaf), and
+ * ccube_gradq_wait then opens once the layer's WEIGHTS are updated.
+ *   weights: nlocal device pointers (this process's ranks), fp32, 16-byte aligned,
+ *            laid out like the gradient buffer (element e <-> element e), at least
+ *            `bytes` long, caller-owned; NULL disables the fused update.
+ * Errors: NOT_INITIALIZED; UNSUPPORTED for world_size 1 (there is no AllReduce
+ * launch to ride on); INVALID_ARG for NULL/misaligned pointers.  While enabled,
+ * ccube_allreduce_tree* accepts only CCUBE_FLOAT32 and count * 4 <= bytes. */
+CCUBE_API ccube_result_t ccube_gradq_set_sgd(void *const *weights, size_t bytes, float alpha);
+
 /* 1 = C1, the root broadcasts chunk k as soon as it is reduced (default,
  * P:L163); 0 = B, the root broadcasts only after all chunks are reduced (P:L119,
  * the paper's baseline "B").  Values are bitwise identical. */
 CCUBE_API ccube_result_t ccube_set_overlap(int on);
 
-/* Channels J per tree (CTA slices of every chunk); all ranks must agree.  0 = the
- * default (CCUBE_CHANNELS env or 8).  `threads` = data threads per CTA (32..256,
+/* Channels J per tree (CTA slices of every chunk); all ranks must agree.  0 = auto
+ * (CCUBE_CHANNELS env, else the most channels whose CTAs are co-resident, capped at
+ * one channel per two 2 KB units of a chunk).  `threads` = data threads per CTA (32..256,
  * multiple of 32; CCUBE_THREADS env, default 256); each CTA adds one control warp. */
 CCUBE_API ccube_result_t ccube_set_channels(int channels);
 CCUBE_API ccube_result_t ccube_set_threads(int threads);
@@ -186,13 +212,14 @@ CCUBE_API const char *ccube_last_error(void);
 typedef struct {
   int initialized, world_size, rank, nlocal, ntrees, channels, threads, overlap, transport;
   size_t chunk_bytes;
-  uint64_t epoch_base[2];
+  uint64_t epoch_base[2];       /* trees 0 and 1 (ROTATED has P trees) */
   int last_channels, last_ctas;
 } ccube_info_t;
 CCUBE_API ccube_result_t ccube_get_info(ccube_info_t *info);
 
 /* The library's own tree builder (host, pure function): parent[v] of tree `tree`
- * (0 or 1) of `kind` for P ranks, -1 at the root. */
+ * (0 for SINGLE, 0..1 for DOUBLE, 0..P-1 for ROTATED) of `kind` for P ranks, -1 at
+ * the root. */
 CCUBE_API ccube_result_t ccube_tree_parents(int P, ccube_tree_kind_t kind, int tree, int *parent);
 
 #ifdef __cplusplus

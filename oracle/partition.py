@@ -8,7 +8,8 @@ Paper basis
   * Two trees "to fully utilize the bandwidth" — no split rule is given.
 
 Readings
-  R4: in the double tree chunk c goes to tree ``c mod 2``.
+  R4: in the double tree chunk c goes to tree ``c mod 2``; with T trees (the
+      rotated set, R17) to tree ``c mod T``.
   R5: the last chunk may be partial; chunk_bytes is a multiple of 16.
   R8: the chunk count is ceil(bytes / chunk_bytes) with chunk_bytes fixed at init;
       eq 4's K_opt is advisory only.
@@ -42,13 +43,13 @@ def chunks(count: int, chunk_bytes: int, elem_size: int) -> List[Tuple[int, int]
 
 
 def tree_of_chunk(c: int, ntrees: int) -> int:
-    """R4: single tree -> 0; double tree -> c mod 2."""
-    return 0 if ntrees == 1 else c % 2
+    """R4: single tree -> 0; double tree -> c mod 2; T trees -> c mod T."""
+    return c % ntrees
 
 
 def tree_local_index(c: int, ntrees: int) -> int:
     """Position of chunk c in its tree's in-order chunk stream."""
-    return c if ntrees == 1 else c // 2
+    return c // ntrees
 
 
 def chunks_of_tree(t: int, K: int, ntrees: int) -> List[int]:

@@ -15,6 +15,11 @@ paper's example 0 <- 2 <- {1, 3} (ranks = N_i - 1 with N4 the root relabelled 0)
 Tree 1 relabels tree 0 by phi(v) = P-1-v for even P (the "flip": tree-0 leaves
 become tree-1 interior nodes) and phi(v) = (v+1) mod P for odd P.
 Children are listed in ascending rank; that order is the combine order (R2).
+
+Rotated set (reading R17): the NVSwitch form of §IV's
+topology-aware trees — P trees, tree t = tree 0 with every rank v
+renamed (v + t) mod P, so every rank holds every tree position exactly once and
+each rank's port carries 2(P-1)/P of the buffer per direction.
 """
 
 from dataclasses import dataclass
@@ -96,10 +101,22 @@ def tree1(P: int) -> Tree:
     return _from_parent(P, parent)
 
 
+def rotated(P: int, t: int) -> Tree:
+    """Tree t of the rotated set (R17): tree 0 with every rank v renamed (v + t) mod P."""
+    t0 = tree0(P)
+    parent = [-1] * P
+    for v in range(P):
+        pv = t0.parent[v]
+        parent[(v + t) % P] = -1 if pv == -1 else (pv + t) % P
+    return _from_parent(P, parent)
+
+
 def trees(P: int, kind: str) -> List[Tree]:
-    """kind = 'single' -> [tree0]; 'double' -> [tree0, tree1]."""
+    """kind = 'single' -> [tree0]; 'double' -> [tree0, tree1]; 'rotated' -> P trees."""
     if kind == "single":
         return [tree0(P)]
     if kind == "double":
         return [tree0(P), tree1(P)]
+    if kind == "rotated":
+        return [rotated(P, t) for t in range(max(P, 1))]
     raise ValueError(kind)

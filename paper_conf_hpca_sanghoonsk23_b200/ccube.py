@@ -30,14 +30,14 @@ ERR_TIMEOUT = -7
 _NAMES = {0: "SUCCESS", -1: "INVALID_ARG", -2: "NOT_INITIALIZED", -3: "ALREADY_INITIALIZED",
           -4: "CUDA", -5: "UNSUPPORTED", -6: "BOOTSTRAP", -7: "TIMEOUT"}
 
-TREE = {"single": 0, "double": 1}
+TREE = {"single": 0, "double": 1, "rotated": 2}
 TRANSPORT = {"auto": 0, "push": 1, "pull": 2}
 DTYPE = {"int32": 0, "float32": 1, "bfloat16": 2}
 
 EXPORTS = [
     "ccube_init", "ccube_register_buffers", "ccube_deregister_buffers", "ccube_allreduce_tree",
     "ccube_allreduce_tree_local", "ccube_gradq_set_layers", "ccube_gradq_wait",
-    "ccube_gradq_wait_local", "ccube_set_overlap", "ccube_set_channels", "ccube_set_threads",
+    "ccube_gradq_wait_local", "ccube_gradq_set_sgd", "ccube_set_overlap", "ccube_set_channels", "ccube_set_threads",
     "ccube_set_trace", "ccube_set_transport", "ccube_finalize", "ccube_last_error", "ccube_get_info",
     "ccube_tree_parents",
 ]
@@ -89,6 +89,7 @@ def lib() -> ctypes.CDLL:
             "ccube_gradq_set_layers": [ctypes.POINTER(sz), i],
             "ccube_gradq_wait": [i, vp],
             "ccube_gradq_wait_local": [i, i, vp],
+            "ccube_gradq_set_sgd": [ctypes.POINTER(vp), sz, ctypes.c_float],
             "ccube_set_overlap": [i],
             "ccube_set_channels": [i],
             "ccube_set_threads": [i],
@@ -252,6 +253,21 @@ def gradq_wait(layer_id: int, stream=None) -> None:
 def gradq_wait_local(local_rank: int, layer_id: int, stream=None) -> None:
     _check(lib().ccube_gradq_wait_local(local_rank, layer_id, _stream_handle(stream)),
            "ccube_gradq_wait_local")
+
+
+def gradq_set_sgd(weights, alpha: float = 0.0) -> None:
+    """Fused SGD update (f2): ``weights`` = one contiguous fp32 CUDA tensor per rank
+    hosted by this process (gradient-buffer layout), or None to disable."""
+    if weights is None:
+        _check(lib().ccube_gradq_set_sgd(None, 0, 0.0), "ccube_gradq_set_sgd")
+        return
+    ws = list(weights)
+    for w in ws:
+        if not w.is_contiguous():
+            raise CCubeError(ERR_INVALID_ARG, "ccube_gradq_set_sgd", "weights must be contiguous")
+    nbytes = min(w.numel() * w.element_size() for w in ws)
+    _check(lib().ccube_gradq_set_sgd(_ptr_array([w.data_ptr() for w in ws]), nbytes, alpha),
+           "ccube_gradq_set_sgd")
 
 
 # ------------------------------------------------------------------------- knobs

@@ -5,7 +5,10 @@
 //            flag(tree, kind, channel) — kind kUpHead0/1: "partial of my k-th chunk
 //            is in your receive plane" written by child slot 0/1 into the parent;
 //            kind kEnq: the Enqueue Semaphore (Fig 9) written by the
-//            parent (or by the root itself) after a fully reduced chunk landed.
+//            parent (or by the root itself) after a fully reduced chunk landed;
+//            kind kUpd: with the fused SGD update (NEXT f2), written by this rank's
+//            own task once its weights of the chunk are updated (the gate then
+//            waits on it instead of kEnq).
 //   recv   : per registered buffer, 2 planes x bytes; child slot s of either tree
 //            writes its partial sum of chunk c at plane s, element offset c*E
 //            (the two trees carry disjoint chunks, so they share the planes).
@@ -24,13 +27,13 @@
 namespace ccube {
 
 constexpr int kMaxRanks = 8;
-constexpr int kMaxChannels = 64;
-constexpr int kMaxTrees = 2;
+constexpr int kMaxChannels = 128;
+constexpr int kMaxTrees = 8;  // ROTATED: one tree per rank
 constexpr int kMaxChildren = 2;
 constexpr int kFlagStride = 64;  // bytes between two counters
 constexpr int kFlagStrideU64 = kFlagStride / 8;
 
-enum FlagKind { kUpHead0 = 0, kUpHead1 = 1, kEnq = 2, kNumFlagKinds = 3 };
+enum FlagKind { kUpHead0 = 0, kUpHead1 = 1, kEnq = 2, kUpd = 3, kNumFlagKinds = 4 };
 
 CCUBE_HD inline size_t flag_offset(int tree, int kind, int ch) {
   return ((static_cast<size_t>(tree) * kNumFlagKinds + kind) * kMaxChannels + ch) * kFlagStride;
@@ -67,9 +70,13 @@ struct TreeParams {
   int self_local;                   // local index of this rank (trace)
   int child_local[kMaxChildren];    // local index of each child, -1 if remote (trace)
   int child_interior[kMaxChildren]; // child has children: its buffer is re-read (DOWN)
+  char *w;                          // own fp32 weights (fused SGD, f2), same layout as buf
+  uint64_t *upd;                    // own "weights updated" counter (channel 0)
 };
 
-enum Role { kRoleUp = 0, kRoleDown = 1 };
+// UPDATE: a leaf's fused-SGD task (f2) — waits for its chunks to land, then
+// w <- w - alpha * g in place (leaves have no DOWN task that reads their result).
+enum Role { kRoleUp = 0, kRoleDown = 1, kRoleUpdate = 2 };
 
 enum { kAllChannels = -1 };  // a pulled leaf's single task covers every channel
 
@@ -96,6 +103,8 @@ struct LaunchArgs {
   uint64_t *trace;            // optional landing trace
   uint32_t trace_kmax;
   int l2_hints;               // 1 = per-stream L2 eviction priorities (keep re-read data)
+  int sgd;                    // 1 = fused SGD update at landing (fp32 only)
+  float sgd_alpha;            // w <- w - sgd_alpha * g
 };
 
 // Kernel launcher (tree_allreduce.cu).  Returns a cudaError_t as int.
@@ -104,6 +113,6 @@ int launch_tree_allreduce(const LaunchArgs &args, int dtype, bool sys_scope, int
 constexpr int kMaxGateCounters = 128;
 int launch_gate(const uint64_t *const *counters, const uint64_t *targets, int n, int *err,
                 uint64_t timeout_ns, bool sys_scope, void *stream);
-int query_max_blocks_per_sm(int dtype, bool sys_scope, int threads, int *blocks);
+int query_max_blocks_per_sm(int dtype, bool sys_scope, bool sgd, int threads, int *blocks);
 
 }  // namespace ccube

@@ -18,6 +18,7 @@
 #include <cstdint>
 #include <cstdio>
 #include <cstdlib>
+#include <algorithm>
 #include <cstring>
 #include <map>
 #include <memory>
@@ -156,21 +157,27 @@ struct Comm {
   size_t chunk_bytes = CCUBE_DEFAULT_CHUNK_BYTES;
   Tree trees[kMaxTrees];
   int channels = 0, threads = 256, overlap = 1;  // channels 0 = auto
-  uint64_t base[kMaxTrees] = {0, 0};
+  int tree_kind = CCUBE_TREE_SINGLE;
+  uint64_t base[kMaxTrees] = {};
   bool have_call = false;
-  uint64_t last_base[kMaxTrees] = {0, 0};
-  uint32_t last_K[kMaxTrees] = {0, 0};
+  uint64_t last_base[kMaxTrees] = {};
+  uint32_t last_K[kMaxTrees] = {};
   uint64_t last_E = 0;
   int last_channels = 0;
   int last_ctas = 0;
   int l2_hints = 1;
+  bool sgd = false;                 // fused SGD update (f2)
+  float sgd_alpha = 0.0f;
+  size_t sgd_bytes = 0;
+  std::vector<char *> sgd_w;        // [nlocal] weights, gradient-buffer layout
+  bool last_sgd = false;
   std::vector<size_t> layer_ends;
   std::vector<char *> flags_local;  // [nlocal]
   std::vector<char *> world_flags;  // [world]
   std::vector<void *> opened_flags;
   int *err_host = nullptr, *err_dev = nullptr;
   std::vector<std::unique_ptr<Registration>> regs;
-  std::map<std::pair<int, int>, TaskTable> tasks;  // (channels, overlap)
+  std::map<std::pair<int, int>, TaskTable> tasks;  // (channels, overlap * 2 + sgd)
   int transport = CCUBE_TRANSPORT_AUTO;
   bool sys_scope = false;
   uint64_t timeout_ns = 10000ull * 1000000ull;
@@ -303,6 +310,8 @@ ccube_result_t build_params(Registration *R) {
         p.child_local[s] = -1;
       }
       p.enq = reinterpret_cast<uint64_t *>(fl + flag_offset(t, kEnq, 0));
+      p.upd = reinterpret_cast<uint64_t *>(fl + flag_offset(t, kUpd, 0));
+      p.w = g.sgd ? g.sgd_w[i] : nullptr;
       const int par = tr.parent[r];
       if (par < 0) {
         p.up_dst = R->bufs[i];  // the root's combine is final
@@ -405,7 +414,7 @@ Registration *find_registration(void *const *bufs, size_t bytes) {
 }
 
 ccube_result_t get_tasks(int channels, int overlap, TaskTable **out) {
-  auto key = std::make_pair(channels, overlap);
+  auto key = std::make_pair(channels, overlap * 2 + (g.sgd ? 1 : 0));
   auto it = g.tasks.find(key);
   if (it != g.tasks.end()) {
     *out = &it->second;
@@ -417,6 +426,9 @@ ccube_result_t get_tasks(int channels, int overlap, TaskTable **out) {
     for (int t = 0; t < g.ntrees; ++t) {
       const Tree &tr = g.trees[t];
       const bool root = tr.parent[r] < 0;
+      if (!root && tr.nchild[r] == 0 && g.sgd)  // a leaf's fused SGD step (f2)
+        for (int j = 0; j < channels; ++j)
+          ts.push_back(Task{(int16_t)i, (int16_t)t, (int16_t)kRoleUpdate, (int16_t)j});
       if (!root && tr.nchild[r] == 0 && edge_is_pull(r, tr.parent[r])) {
         ts.push_back(Task{(int16_t)i, (int16_t)t, (int16_t)kRoleUp, (int16_t)kAllChannels});
         continue;
@@ -454,6 +466,7 @@ int count_tasks(int channels, int overlap) {
     for (int t = 0; t < g.ntrees; ++t) {
       const Tree &tr = g.trees[t];
       const bool root = tr.parent[r] < 0;
+      if (!root && tr.nchild[r] == 0 && g.sgd) n += channels;
       if (!root && tr.nchild[r] == 0 && edge_is_pull(r, tr.parent[r])) {
         n += 1;
         continue;
@@ -479,6 +492,13 @@ ccube_result_t allreduce_impl(void *const *bufs, size_t count, ccube_dtype_t dty
   }
   const int es = elem_size(dtype);
   if (count > (~0ull) / 4) return fail(CCUBE_ERR_INVALID_ARG, "count too large");
+  if (g.sgd && g.world > 1 && count > 0) {
+    if (dtype != CCUBE_FLOAT32)
+      return fail(CCUBE_ERR_INVALID_ARG, "the fused SGD update needs fp32 gradients");
+    if (count * 4 > g.sgd_bytes)
+      return fail(CCUBE_ERR_INVALID_ARG, "count %zu exceeds the registered weights (%zu bytes)",
+                  count, g.sgd_bytes);
+  }
   if (g.world == 1 || count == 0) return CCUBE_SUCCESS;
   const size_t bytes = count * es;
   Registration *R = find_registration(bufs, bytes);
@@ -490,11 +510,11 @@ ccube_result_t allreduce_impl(void *const *bufs, size_t count, ccube_dtype_t dty
 
   // all CTAs spin on each other: they must be co-resident
   const int cta_threads = g.threads + 32;  // data warps + the control warp
-  auto key = std::make_pair((int)dtype, cta_threads);
+  auto key = std::make_pair((int)dtype * 2 + (g.sgd ? 1 : 0), cta_threads);
   if (!g.max_blocks.count(key)) {
     int b = 0;
     const int rc =
-        query_max_blocks_per_sm(dtype, g.sys_scope, cta_threads, &b);
+        query_max_blocks_per_sm(dtype, g.sys_scope, g.sgd, cta_threads, &b);
     if (rc != cudaSuccess)
       return fail(CCUBE_ERR_CUDA, "occupancy query failed: %s",
                   cudaGetErrorString(static_cast<cudaError_t>(rc)));
@@ -502,9 +522,15 @@ ccube_result_t allreduce_impl(void *const *bufs, size_t count, ccube_dtype_t dty
   }
   const int cap = g.max_blocks[key] * g.sm_count;
   int J = g.channels;
-  if (J == 0) {  // auto: the most channels whose CTAs all fit at once
+  if (J == 0) {  // auto: the most channels whose CTAs all fit at once ...
     J = 1;
     while (J < CCUBE_MAX_CHANNELS && count_tasks(J + 1, g.overlap) <= cap) ++J;
+    // ... but at least two 2 KB units per channel and chunk: a small buffer gets
+    // few channels, so few CTAs take part in the handshakes (latency)
+    const uint64_t first = bytes < g.chunk_bytes ? bytes : g.chunk_bytes;
+    const uint64_t units = (first + 2047) / 2048;
+    const int jmax = units / 2 > 1 ? static_cast<int>(units / 2) : 1;
+    if (J > jmax) J = jmax;
   }
 
   LaunchArgs a;
@@ -513,12 +539,8 @@ ccube_result_t allreduce_impl(void *const *bufs, size_t count, ccube_dtype_t dty
   a.elems_per_chunk = static_cast<uint32_t>(E);
   a.ntrees = g.ntrees;
   a.nchannels = J;
-  if (g.ntrees == 1) {
-    a.K[0] = static_cast<uint32_t>(K);
-  } else {
-    a.K[0] = static_cast<uint32_t>((K + 1) / 2);
-    a.K[1] = static_cast<uint32_t>(K / 2);
-  }
+  for (int t = 0; t < g.ntrees; ++t)  // chunk c travels on tree c mod T (R4)
+    a.K[t] = static_cast<uint32_t>(K > static_cast<uint64_t>(t) ? (K - t + g.ntrees - 1) / g.ntrees : 0);
   for (int t = 0; t < g.ntrees; ++t) a.base[t] = g.base[t];
   a.overlap = g.overlap;
   a.timeout_ns = g.timeout_ns;
@@ -526,6 +548,8 @@ ccube_result_t allreduce_impl(void *const *bufs, size_t count, ccube_dtype_t dty
   a.trace = g.trace;
   a.trace_kmax = static_cast<uint32_t>(g.trace_kmax);
   a.l2_hints = g.l2_hints;
+  a.sgd = g.sgd ? 1 : 0;
+  a.sgd_alpha = g.sgd_alpha;
   a.params = R->d_params;
 
   TaskTable *tt = nullptr;
@@ -543,6 +567,7 @@ ccube_result_t allreduce_impl(void *const *bufs, size_t count, ccube_dtype_t dty
   g.have_call = true;
   g.last_E = E;
   g.last_channels = J;
+  g.last_sgd = g.sgd;
   g.last_ctas = tt->n;
   for (int t = 0; t < g.ntrees; ++t) {
     g.last_base[t] = g.base[t];
@@ -562,47 +587,56 @@ ccube_result_t gradq_wait_impl(int local_rank, int layer_id, void *stream) {
                 g.layer_ends.size());
   if (g.world == 1 || !g.have_call) return CCUBE_SUCCESS;
   // LCT[l] = ceil(end_l / E) chunks (R9, R10); tree t needs its share (R4)
-  const uint64_t total_K = g.ntrees == 1 ? g.last_K[0] : g.last_K[0] + g.last_K[1];
+  uint64_t total_K = 0;
+  for (int t = 0; t < g.ntrees; ++t) total_K += g.last_K[t];
   uint64_t lct = (g.layer_ends[layer_id] + g.last_E - 1) / g.last_E;
   if (lct > total_K) lct = total_K;
-  uint64_t need[kMaxTrees] = {lct, 0};
-  if (g.ntrees == 2) {
-    need[0] = (lct + 1) / 2;
-    need[1] = lct / 2;
-  }
+  // tree t carries chunks t, t+T, ...: layer l needs ceil((LCT - t) / T) of them
+  uint64_t need[kMaxTrees] = {};
+  for (int t = 0; t < g.ntrees; ++t)
+    need[t] = lct > static_cast<uint64_t>(t) ? (lct - t + g.ntrees - 1) / g.ntrees : 0;
   std::vector<const uint64_t *> ctr;
   std::vector<uint64_t> tgt;
   for (int t = 0; t < g.ntrees; ++t) {
     if (need[t] == 0) continue;
     for (int j = 0; j < g.last_channels; ++j) {
-      ctr.push_back(reinterpret_cast<const uint64_t *>(g.flags_local[local_rank] +
-                                                       flag_offset(t, kEnq, j)));
+      // with the fused update the gate opens once the WEIGHTS of the chunk are updated
+      ctr.push_back(reinterpret_cast<const uint64_t *>(
+          g.flags_local[local_rank] + flag_offset(t, g.last_sgd ? kUpd : kEnq, j)));
       tgt.push_back(g.last_base[t] + need[t]);
     }
   }
-  if (ctr.empty()) return CCUBE_SUCCESS;
+  // waits are idempotent ">=" checks, so they may be split into batches freely
+  size_t done = 0;
   if (g.use_memop) {
     load_driver();
-    if (g_drv.batchMemOp) {
-      std::vector<CUstreamBatchMemOpParams> ops(ctr.size());
-      for (size_t i = 0; i < ctr.size(); ++i) {
+    while (g_drv.batchMemOp && done < ctr.size()) {
+      const size_t n = std::min(ctr.size() - done, static_cast<size_t>(kMaxGateCounters));
+      std::vector<CUstreamBatchMemOpParams> ops(n);
+      for (size_t i = 0; i < n; ++i) {
         memset(&ops[i], 0, sizeof ops[i]);
         ops[i].waitValue.operation = CU_STREAM_MEM_OP_WAIT_VALUE_64;
-        ops[i].waitValue.address = reinterpret_cast<CUdeviceptr>(ctr[i]);
-        ops[i].waitValue.value64 = tgt[i];
+        ops[i].waitValue.address = reinterpret_cast<CUdeviceptr>(ctr[done + i]);
+        ops[i].waitValue.value64 = tgt[done + i];
         ops[i].waitValue.flags = CU_STREAM_WAIT_VALUE_GEQ;
       }
-      const CUresult cr = g_drv.batchMemOp(static_cast<CUstream>(stream),
-                                           static_cast<unsigned>(ops.size()), ops.data(), 0);
-      if (cr == CUDA_SUCCESS) return CCUBE_SUCCESS;
+      if (g_drv.batchMemOp(static_cast<CUstream>(stream), static_cast<unsigned>(n), ops.data(),
+                           0) != CUDA_SUCCESS)
+        break;
+      done += n;
     }
+    if (done == ctr.size()) return CCUBE_SUCCESS;
     g.use_memop = false;  // fall back to the spin-gate kernel from now on
   }
-  const int rc = launch_gate(ctr.data(), tgt.data(), static_cast<int>(ctr.size()), g.err_dev,
-                             g.timeout_ns, g.sys_scope, stream);
-  if (rc != cudaSuccess)
-    return fail(CCUBE_ERR_CUDA, "gate launch failed: %s",
-                cudaGetErrorString(static_cast<cudaError_t>(rc)));
+  while (done < ctr.size()) {
+    const int n = static_cast<int>(std::min(ctr.size() - done, static_cast<size_t>(kMaxGateCounters)));
+    const int rc = launch_gate(ctr.data() + done, tgt.data() + done, n, g.err_dev, g.timeout_ns,
+                               g.sys_scope, stream);
+    if (rc != cudaSuccess)
+      return fail(CCUBE_ERR_CUDA, "gate launch failed: %s",
+                  cudaGetErrorString(static_cast<cudaError_t>(rc)));
+    done += n;
+  }
   return CCUBE_SUCCESS;
 }
 
@@ -651,7 +685,8 @@ ccube_result_t ccube_init(const ccube_world_t *world, ccube_tree_kind_t tree_kin
   if (world->rank < 0 || world->rank >= P || world->rank % world->nlocal)
     return fail(CCUBE_ERR_INVALID_ARG, "rank %d must be a multiple of nlocal in [0, %d)",
                 world->rank, P);
-  if (tree_kind != CCUBE_TREE_SINGLE && tree_kind != CCUBE_TREE_DOUBLE)
+  if (tree_kind != CCUBE_TREE_SINGLE && tree_kind != CCUBE_TREE_DOUBLE &&
+      tree_kind != CCUBE_TREE_ROTATED)
     return fail(CCUBE_ERR_INVALID_ARG, "bad tree kind %d", (int)tree_kind);
   if (world->nlocal < P && !world->allgather)
     return fail(CCUBE_ERR_INVALID_ARG, "allgather callback required when nlocal < world_size");
@@ -676,7 +711,8 @@ ccube_result_t ccube_init(const ccube_world_t *world, ccube_tree_kind_t tree_kin
   g.proc = world->rank / world->nlocal;
   g.allgather = world->allgather;
   g.ctx = world->ctx;
-  g.ntrees = tree_kind == CCUBE_TREE_DOUBLE ? 2 : 1;
+  g.tree_kind = tree_kind;
+  g.ntrees = num_trees(P, tree_kind);
   g.chunk_bytes = chunk_bytes;
   g.channels = channels;
   g.threads = threads;
@@ -686,7 +722,7 @@ ccube_result_t ccube_init(const ccube_world_t *world, ccube_tree_kind_t tree_kin
   g.sys_scope = g.nproc > 1;
   g.timeout_ns = static_cast<uint64_t>(env_int("CCUBE_WATCHDOG_MS", 10000)) * 1000000ull;
   g.use_memop = env_int("CCUBE_GATE_KERNEL", 0) == 0;
-  for (int t = 0; t < g.ntrees; ++t) build_tree(P, t, &g.trees[t]);
+  for (int t = 0; t < g.ntrees; ++t) build_tree(P, tree_kind, t, &g.trees[t]);
 
   // (i) config agreement — host only, so it also runs (and can be tested) without a GPU
   Hello mine;
@@ -849,6 +885,32 @@ ccube_result_t ccube_set_overlap(int on) {
   return CCUBE_SUCCESS;
 }
 
+ccube_result_t ccube_gradq_set_sgd(void *const *weights, size_t bytes, float alpha) {
+  std::lock_guard<std::mutex> lk(g_mu);
+  if (!g.init) return fail(CCUBE_ERR_NOT_INITIALIZED, "ccube_init has not been called");
+  if (!weights) {
+    g.sgd = false;
+    g.sgd_w.clear();
+    g.sgd_bytes = 0;
+  } else {
+    if (g.world < 2)
+      return fail(CCUBE_ERR_UNSUPPORTED, "the fused SGD update rides on the AllReduce (P >= 2)");
+    if (bytes == 0 || bytes % 4) return fail(CCUBE_ERR_INVALID_ARG, "bad weight bytes %zu", bytes);
+    for (int i = 0; i < g.nlocal; ++i) {
+      if (!weights[i]) return fail(CCUBE_ERR_INVALID_ARG, "weights[%d] is NULL", i);
+      if (reinterpret_cast<uintptr_t>(weights[i]) % 16)
+        return fail(CCUBE_ERR_INVALID_ARG, "weights[%d] is not 16-byte aligned", i);
+    }
+    g.sgd = true;
+    g.sgd_alpha = alpha;
+    g.sgd_bytes = bytes;
+    g.sgd_w.assign(g.nlocal, nullptr);
+    for (int i = 0; i < g.nlocal; ++i) g.sgd_w[i] = static_cast<char *>(weights[i]);
+  }
+  for (auto &R : g.regs) CC_TRY(build_params(R.get()));  // weights are per-rank params
+  return CCUBE_SUCCESS;
+}
+
 ccube_result_t ccube_set_channels(int channels) {
   std::lock_guard<std::mutex> lk(g_mu);
   if (!g.init) return fail(CCUBE_ERR_NOT_INITIALIZED, "ccube_init has not been called");
@@ -940,10 +1002,12 @@ ccube_result_t ccube_get_info(ccube_info_t *info) {
 
 ccube_result_t ccube_tree_parents(int P, ccube_tree_kind_t kind, int tree, int *parent) {
   if (P < 1 || P > kTreeMaxP || !parent) return fail(CCUBE_ERR_INVALID_ARG, "bad P or parent");
-  if (tree < 0 || tree > (kind == CCUBE_TREE_DOUBLE ? 1 : 0))
+  if (kind != CCUBE_TREE_SINGLE && kind != CCUBE_TREE_DOUBLE && kind != CCUBE_TREE_ROTATED)
+    return fail(CCUBE_ERR_INVALID_ARG, "bad tree kind %d", (int)kind);
+  if (tree < 0 || tree >= num_trees(P, kind))
     return fail(CCUBE_ERR_INVALID_ARG, "bad tree index %d", tree);
   Tree t;
-  build_tree(P, tree, &t);
+  build_tree(P, kind, tree, &t);
   for (int v = 0; v < P; ++v) parent[v] = t.parent[v];
   return CCUBE_SUCCESS;
 }

@@ -244,9 +244,11 @@ constexpr uint32_t kUnit = 2048;
 struct Geo {
   uint64_t Eb;       // chunk bytes
   uint64_t nbytes;   // buffer bytes
-  uint32_t T, t;     // trees, this tree
+  uint64_t stride;   // bytes between consecutive chunks of this tree (T * Eb)
+  uint64_t first;    // byte offset of this tree's chunk 0 (t * Eb)
   uint32_t J, j;     // channels, this channel
   uint32_t K;        // tree-local chunks
+  uint32_t q, r;     // split of a full chunk's units: q each, one more for r channels
 };
 
 struct Slice {
@@ -259,26 +261,33 @@ __device__ __forceinline__ Geo make_geo(const LaunchArgs &a, int t, int j) {
   Geo g;
   g.Eb = static_cast<uint64_t>(a.elems_per_chunk) * ES;
   g.nbytes = a.count * ES;
-  g.T = a.ntrees;
-  g.t = t;
+  g.stride = g.Eb * a.ntrees;
+  g.first = g.Eb * t;
   g.J = a.nchannels;
   g.j = j;
   g.K = a.K[t];
+  const uint32_t n = static_cast<uint32_t>((g.Eb + kUnit - 1) / kUnit);
+  g.q = n / g.J;
+  g.r = n % g.J;
   return g;
 }
 
-// f(x) = #{m in [0, x) : m mod J < r}
-__device__ __forceinline__ uint32_t extra_before(uint32_t x, uint32_t J, uint32_t r) {
-  return (x / J) * r + min(x % J, r);
-}
-
-__device__ __forceinline__ Slice slice_of(const Geo &g, uint32_t k) {
-  const uint64_t c0 = (static_cast<uint64_t>(k) * g.T + g.t) * g.Eb;
+// Slice of channel j in the chunk at byte offset c0, whose tree-local index k has
+// c = k mod J.  Channel i gets q units plus one iff (i + c) mod J < r; channel j
+// starts after f(c + j) - f(c) extra units, f(x) = #{m < x : m mod J < r}.  With
+// c, j < J every term is a compare (no division) except for the short last chunk.
+__device__ __forceinline__ Slice slice_at(const Geo &g, uint32_t c, uint64_t c0) {
   const uint64_t clen = min(g.Eb, g.nbytes - c0);
-  const uint32_t n = static_cast<uint32_t>((clen + kUnit - 1) / kUnit);
-  const uint32_t q = n / g.J, r = n % g.J, c = k % g.J;
-  const uint32_t u0 = g.j * q + extra_before(c + g.j, g.J, r) - extra_before(c, g.J, r);
-  const uint32_t nu = q + ((g.j + c) % g.J < r ? 1u : 0u);
+  uint32_t q = g.q, r = g.r;
+  if (clen < g.Eb) {  // the short last chunk has its own split
+    const uint32_t n = static_cast<uint32_t>((clen + kUnit - 1) / kUnit);
+    q = n / g.J;
+    r = n % g.J;
+  }
+  const uint32_t x = c + g.j;                                // < 2J
+  const uint32_t fx = x < g.J ? min(x, r) : r + min(x - g.J, r);
+  const uint32_t u0 = g.j * q + fx - min(c, r);
+  const uint32_t nu = q + ((x < g.J ? x : x - g.J) < r ? 1u : 0u);
   const uint64_t lo = min(static_cast<uint64_t>(u0) * kUnit, clen);
   const uint64_t hi = min(static_cast<uint64_t>(u0 + nu) * kUnit, clen);
   Slice s;
@@ -290,36 +299,44 @@ __device__ __forceinline__ Slice slice_of(const Geo &g, uint32_t k) {
 // A data warp's walk over its blocks: blocks of `seg` bytes tile each chunk's
 // slice; warp w of W takes blocks w, w+W, ... of the concatenation over chunks,
 // so a warp's blocks are in chunk order (the readiness check and the base
-// address of a block are warp-uniform).
+// address of a block are warp-uniform).  Advanced without divisions.
 struct BlockIter {
   uint32_t k;    // chunk (tree-local); K = finished
+  uint32_t c;    // k mod J
+  uint64_t c0;   // byte offset of chunk k
   uint32_t s;    // block inside the chunk's slice
   uint32_t nb;   // blocks in this chunk's slice
   Slice sl;      // this chunk's slice
 };
 
-__device__ __forceinline__ void iter_settle(const Geo &g, uint32_t seg, BlockIter &it) {
+template <uint32_t SEG>
+__device__ __forceinline__ void iter_settle(const Geo &g, BlockIter &it) {
   while (it.k < g.K && it.s >= it.nb) {
     it.s -= it.nb;
     if (++it.k < g.K) {
-      it.sl = slice_of(g, it.k);
-      it.nb = (it.sl.len + seg - 1) / seg;
+      it.c = it.c + 1 == g.J ? 0 : it.c + 1;
+      it.c0 += g.stride;
+      it.sl = slice_at(g, it.c, it.c0);
+      it.nb = (it.sl.len + SEG - 1) / SEG;
     }
   }
 }
 
-__device__ __forceinline__ BlockIter iter_begin(const Geo &g, uint32_t seg, uint32_t w) {
+template <uint32_t SEG>
+__device__ __forceinline__ BlockIter iter_begin(const Geo &g, uint32_t w) {
   BlockIter it;
   it.k = 0;
+  it.c = 0;
+  it.c0 = g.first;
   it.s = w;
   it.nb = 0;
   it.sl.off = 0;
   it.sl.len = 0;
   if (g.K > 0) {
-    it.sl = slice_of(g, 0);
-    it.nb = (it.sl.len + seg - 1) / seg;
+    it.sl = slice_at(g, 0, it.c0);
+    it.nb = (it.sl.len + SEG - 1) / SEG;
   }
-  iter_settle(g, seg, it);
+  iter_settle<SEG>(g, it);
   return it;
 }
 
@@ -329,11 +346,32 @@ struct Endpoints {
   char *dst[kMaxIn];
   int nin, nout;
   uint32_t keep;  // bit q: dst[q] is re-read later in this launch (L2 evict_last)
+  bool sgd;       // this task also applies the fused SGD step to my weights (f2)
+  char *w;        // my weights
+  const char *gfinal;  // where my final gradient sits (ragged-tail scalar path)
 };
+
+// The task that applies rank v's fused SGD step (f2) is the one that handles v's
+// final gradient anyway: the root's UP task (it computes it), an interior rank's
+// DOWN task (it reads it to forward it), a leaf's UPDATE task.
+__device__ __forceinline__ bool does_sgd(const LaunchArgs &a, const TreeParams &p, int role) {
+  if (!a.sgd) return false;
+  if (role == kRoleUpdate) return true;
+  return role == kRoleUp ? p.is_root != 0 : p.is_root == 0;
+}
 
 __device__ __forceinline__ Endpoints endpoints(const LaunchArgs &a, const TreeParams &p, int role) {
   Endpoints e;
   e.keep = 0;
+  e.sgd = does_sgd(a, p, role);
+  e.w = p.w;
+  e.gfinal = p.buf;
+  if (role == kRoleUpdate) {
+    e.nin = 1;
+    e.src[0] = p.buf;
+    e.nout = 0;
+    return e;
+  }
   if (role == kRoleUp) {
     e.nin = 1 + p.nchild;
     for (int q = 0; q < e.nin; ++q) e.src[q] = p.up_src[q];
@@ -417,6 +455,8 @@ __device__ __forceinline__ void publish(const LaunchArgs &a, const TreeParams &p
   const int stride = j * kFlagStrideU64;
   const uint64_t v = base + d;
   fence_release<SYS>();
+  if (does_sgd(a, p, role)) st_relaxed<SYS>(p.upd + stride, v);  // my weights updated
+  if (role == kRoleUpdate) return;
   if (role == kRoleUp && !p.is_root) {
     st_relaxed<SYS>(p.head_out + stride, v);
     return;
@@ -544,6 +584,7 @@ __device__ void control_warp(const LaunchArgs &a, const TreeParams &p, int role,
       if (lane == 0) {
         *reinterpret_cast<volatile int *>(&sh.abort) = 1;
         st_relaxed<SYS>(p.enq + stride, ~0ull);  // release gradient-queue waiters
+        st_relaxed<SYS>(p.upd + stride, ~0ull);
       }
       return;
     }
@@ -554,7 +595,20 @@ __device__ void control_warp(const LaunchArgs &a, const TreeParams &p, int role,
 // One data warp's stream: blocks of 32*U vectors (512*U bytes), see BlockIter.
 // Lane l handles vectors l + 32u, u < U, of a block: U loads per source in
 // flight, then the fixed-order combine and 128-bit stores to every destination.
-template <int DT, int NIN, int NOUT, int U>
+// SGD (f2, fp32 only): the block's final gradient r also updates my weights,
+// w <- w - alpha * r, as two IEEE-rounded operations (no FMA contraction; the
+// oracle's reading R18) — one extra load and store stream, no extra pass.
+__device__ __forceinline__ float sgd1(float w, float g, float alpha) {
+  return __fsub_rn(w, __fmul_rn(alpha, g));
+}
+__device__ __forceinline__ uint4 sgd4(const uint4 &w, const uint4 &g, float alpha) {
+  return make_uint4(__float_as_uint(sgd1(__uint_as_float(w.x), __uint_as_float(g.x), alpha)),
+                    __float_as_uint(sgd1(__uint_as_float(w.y), __uint_as_float(g.y), alpha)),
+                    __float_as_uint(sgd1(__uint_as_float(w.z), __uint_as_float(g.z), alpha)),
+                    __float_as_uint(sgd1(__uint_as_float(w.w), __uint_as_float(g.w), alpha)));
+}
+
+template <int DT, int NIN, int NOUT, int U, bool SGD>
 __device__ void lsu_stream(const LaunchArgs &a, const Endpoints &e, int t, int j, int w, int W,
                            Shared &sh) {
   constexpr int ES = DT == kBFloat16 ? 2 : 4;
@@ -564,18 +618,19 @@ __device__ void lsu_stream(const LaunchArgs &a, const Endpoints &e, int t, int j
   uint64_t ready = 0;
   uint32_t done_reported = 0;
   const L2Pol pol = make_pol(a.l2_hints);
-  uint64_t dpol[NOUT];
+  const float alpha = a.sgd_alpha;
+  uint64_t dpol[NOUT > 0 ? NOUT : 1];
 #pragma unroll
   for (int q = 0; q < NOUT; ++q) dpol[q] = (e.keep >> q) & 1u ? pol.last : pol.first;
-  BlockIter it = iter_begin(g, kSeg, w);
+  BlockIter it = iter_begin<kSeg>(g, w);
   while (it.k < g.K) {
     const uint32_t k = it.k;
     if (k >= ready) {
       uint64_t r = 0;
-      if (lane == 0) {
-        do {
-          r = ld_acquire_cta(&sh.ready);
-        } while (r <= k && !*reinterpret_cast<volatile int *>(&sh.abort));
+      if (lane == 0) {  // upstream not there yet: back off so busy warps get the issue slots
+        while ((r = ld_acquire_cta(&sh.ready)) <= k &&
+               !*reinterpret_cast<volatile int *>(&sh.abort))
+          __nanosleep(64);
       }
       r = __shfl_sync(0xffffffffu, r, 0);
       if (r <= k) return;  // aborted
@@ -586,16 +641,18 @@ __device__ void lsu_stream(const LaunchArgs &a, const Endpoints &e, int t, int j
     const uint32_t len = min(kSeg, it.sl.len - b0);
     const uint32_t nvec = len / 16;
     uint4 x[U][NIN];
+    uint4 wv[SGD ? U : 1];
 #pragma unroll
     for (int u = 0; u < U; ++u) {
       if (lane + 32u * u < nvec) {
 #pragma unroll
         for (int q = 0; q < NIN; ++q)
           x[u][q] = ld_hint(e.src[q] + off + lane * 16 + 512u * u, pol.first);
+        if constexpr (SGD) wv[u] = ld_hint(e.w + off + lane * 16 + 512u * u, pol.first);
       }
     }
     it.s += W;  // advance while the loads are in flight (the loop is latency bound)
-    iter_settle(g, kSeg, it);
+    iter_settle<kSeg>(g, it);
 #pragma unroll
     for (int u = 0; u < U; ++u) {
       if (lane + 32u * u < nvec) {
@@ -603,10 +660,21 @@ __device__ void lsu_stream(const LaunchArgs &a, const Endpoints &e, int t, int j
 #pragma unroll
         for (int q = 0; q < NOUT; ++q)
           st_hint(e.dst[q] + off + lane * 16 + 512u * u, r, dpol[q]);
+        if constexpr (SGD)
+          st_hint(e.w + off + lane * 16 + 512u * u, sgd4(wv[u], r, alpha), pol.first);
       }
     }
-    if (len & 15u)  // ragged end of the buffer (< 16 bytes, last block only)
-      combine_scalar<DT>(e.src, NIN, e.dst, NOUT, off + (len & ~15u), len & 15u);
+    if (len & 15u) {  // ragged end of the buffer (< 16 bytes, last block only)
+      const uint64_t o = off + (len & ~15u);
+      if (NOUT > 0) combine_scalar<DT>(e.src, NIN, e.dst, NOUT, o, len & 15u);
+      if constexpr (SGD) {
+        __syncwarp();  // the final values written just above (same lanes) come first
+        for (uint32_t x4 = lane; x4 < (len & 15u) / 4; x4 += 32) {
+          float *wp = reinterpret_cast<float *>(e.w + o) + x4;
+          *wp = sgd1(*wp, reinterpret_cast<const float *>(e.gfinal + o)[x4], alpha);
+        }
+      }
+    }
     if (it.k > done_reported) {
       __syncwarp();  // every lane's stores precede the release
       if (lane == 0) st_release_cta(&sh.done[w], it.k);
@@ -619,34 +687,48 @@ __device__ void lsu_stream(const LaunchArgs &a, const Endpoints &e, int t, int j
   }
 }
 
-template <int DT, int NIN>
+template <int DT, int NIN, bool SGD>
 __device__ __forceinline__ void lsu_nout(const LaunchArgs &a, const Endpoints &e, int t, int j,
                                          int w, int W, Shared &sh) {
   constexpr int U = NIN == 1 ? 8 : 4;  // block = 4 KB (copies) or 2 KB (combines)
+  if constexpr (SGD && DT == kFloat32 && NIN <= 2) {
+    if (e.sgd) {  // root UP (NIN 2), interior DOWN and leaf UPDATE (NIN 1); U = 4 (2 KB)
+      switch (e.nout) {
+        case 0: lsu_stream<DT, NIN, 0, 4, true>(a, e, t, j, w, W, sh); return;
+        case 1: lsu_stream<DT, NIN, 1, 4, true>(a, e, t, j, w, W, sh); return;
+        default: lsu_stream<DT, NIN, 2, 4, true>(a, e, t, j, w, W, sh); return;
+      }
+    }
+  }
   switch (e.nout) {
-    case 1: lsu_stream<DT, NIN, 1, U>(a, e, t, j, w, W, sh); break;
-    case 2: lsu_stream<DT, NIN, 2, U>(a, e, t, j, w, W, sh); break;
-    default: lsu_stream<DT, NIN, 3, U>(a, e, t, j, w, W, sh); break;
+    case 1: lsu_stream<DT, NIN, 1, U, false>(a, e, t, j, w, W, sh); break;
+    case 2: lsu_stream<DT, NIN, 2, U, false>(a, e, t, j, w, W, sh); break;
+    default: lsu_stream<DT, NIN, 3, U, false>(a, e, t, j, w, W, sh); break;
   }
 }
 
-template <int DT>
+template <int DT, bool SGD>
 __device__ void data_warp(const LaunchArgs &a, const TreeParams &p, int role, int t, int j,
-                              int w, int W, Shared &sh) {
-  const Endpoints e = endpoints(a, p, role);
-  if (e.nout == 0) {  // nothing to write (cannot happen for scheduled tasks)
+                          int w, int W, Shared &sh) {
+  Endpoints e = endpoints(a, p, role);
+  if (!SGD) e.sgd = false;
+  if (e.nout == 0 && !e.sgd) {  // nothing to write (cannot happen for scheduled tasks)
     if ((threadIdx.x & 31) == 0) st_release_cta(&sh.done[w], a.K[t]);
     return;
   }
   switch (e.nin) {
-    case 1: lsu_nout<DT, 1>(a, e, t, j, w, W, sh); break;
-    case 2: lsu_nout<DT, 2>(a, e, t, j, w, W, sh); break;
-    default: lsu_nout<DT, 3>(a, e, t, j, w, W, sh); break;
+    case 1: lsu_nout<DT, 1, SGD>(a, e, t, j, w, W, sh); break;
+    case 2: lsu_nout<DT, 2, SGD>(a, e, t, j, w, W, sh); break;
+    default: lsu_nout<DT, 3, SGD>(a, e, t, j, w, W, sh); break;
   }
 }
 
-template <int DT, bool SYS>
-__global__ void __launch_bounds__(kMaxThreads, kMinBlocksPerSm) tree_allreduce_kernel(const LaunchArgs a) {
+// SGD = the fp32 variant with the fused update (f2); the plain kernels do not carry
+// its code (register pressure).
+// MAXT = the CTA size bound: 288 (8 data warps) or 256 (7 data warps, which leaves
+// ptxas 128 registers per thread at two CTAs per SM instead of 96).
+template <int DT, bool SYS, bool SGD, int MAXT>
+__global__ void __launch_bounds__(MAXT, kMinBlocksPerSm) tree_allreduce_kernel(const LaunchArgs a) {
   __shared__ Shared sh;
   const Task task = a.tasks[blockIdx.x];
   const TreeParams &p = a.params[task.local_rank * a.ntrees + task.tree];
@@ -665,7 +747,7 @@ __global__ void __launch_bounds__(kMaxThreads, kMinBlocksPerSm) tree_allreduce_k
   if (warp == 0)
     control_warp<SYS>(a, p, task.role, task.tree, task.channel, W, sh);
   else
-    data_warp<DT>(a, p, task.role, task.tree, task.channel, warp - 1, W, sh);
+    data_warp<DT, SGD>(a, p, task.role, task.tree, task.channel, warp - 1, W, sh);
 }
 
 struct GateArgs {
@@ -692,15 +774,20 @@ __global__ void gate_kernel(const GateArgs g) {
   }
 }
 
-template <int DT, bool SYS>
+template <int DT, bool SYS, bool SGD>
 int launch_t(const LaunchArgs &a, int grid, int threads, cudaStream_t s) {
-  tree_allreduce_kernel<DT, SYS><<<grid, threads, 0, s>>>(a);
+  if (threads <= 256)
+    tree_allreduce_kernel<DT, SYS, SGD, 256><<<grid, threads, 0, s>>>(a);
+  else
+    tree_allreduce_kernel<DT, SYS, SGD, kMaxThreads><<<grid, threads, 0, s>>>(a);
   return static_cast<int>(cudaGetLastError());
 }
 
-template <int DT, bool SYS>
-const void *kernel_ptr() {
-  return reinterpret_cast<const void *>(tree_allreduce_kernel<DT, SYS>);
+template <int DT, bool SYS, bool SGD>
+const void *kernel_ptr(int threads) {
+  if (threads <= 256)
+    return reinterpret_cast<const void *>(tree_allreduce_kernel<DT, SYS, SGD, 256>);
+  return reinterpret_cast<const void *>(tree_allreduce_kernel<DT, SYS, SGD, kMaxThreads>);
 }
 
 }  // namespace
@@ -710,16 +797,21 @@ int launch_tree_allreduce(const LaunchArgs &args, int dtype, bool sys_scope, int
   if (threads > kMaxThreads || threads < 64 || threads % 32 || threads / 32 - 1 > kMaxDataWarps)
     return cudaErrorInvalidValue;
   cudaStream_t s = static_cast<cudaStream_t>(stream);
+  if (args.sgd) {
+    if (dtype != kFloat32) return cudaErrorInvalidValue;
+    return sys_scope ? launch_t<kFloat32, true, true>(args, grid, threads, s)
+                     : launch_t<kFloat32, false, true>(args, grid, threads, s);
+  }
   switch (dtype) {
     case kInt32:
-      return sys_scope ? launch_t<kInt32, true>(args, grid, threads, s)
-                       : launch_t<kInt32, false>(args, grid, threads, s);
+      return sys_scope ? launch_t<kInt32, true, false>(args, grid, threads, s)
+                       : launch_t<kInt32, false, false>(args, grid, threads, s);
     case kFloat32:
-      return sys_scope ? launch_t<kFloat32, true>(args, grid, threads, s)
-                       : launch_t<kFloat32, false>(args, grid, threads, s);
+      return sys_scope ? launch_t<kFloat32, true, false>(args, grid, threads, s)
+                       : launch_t<kFloat32, false, false>(args, grid, threads, s);
     case kBFloat16:
-      return sys_scope ? launch_t<kBFloat16, true>(args, grid, threads, s)
-                       : launch_t<kBFloat16, false>(args, grid, threads, s);
+      return sys_scope ? launch_t<kBFloat16, true, false>(args, grid, threads, s)
+                       : launch_t<kBFloat16, false, false>(args, grid, threads, s);
     default:
       return cudaErrorInvalidValue;
   }
@@ -745,18 +837,23 @@ int launch_gate(const uint64_t *const *counters, const uint64_t *targets, int n,
   return static_cast<int>(cudaGetLastError());
 }
 
-int query_max_blocks_per_sm(int dtype, bool sys_scope, int threads, int *blocks) {
+int query_max_blocks_per_sm(int dtype, bool sys_scope, bool sgd, int threads, int *blocks) {
   const void *fn = nullptr;
-  switch (dtype) {
-    case kInt32:
-      fn = sys_scope ? kernel_ptr<kInt32, true>() : kernel_ptr<kInt32, false>();
-      break;
-    case kFloat32:
-      fn = sys_scope ? kernel_ptr<kFloat32, true>() : kernel_ptr<kFloat32, false>();
-      break;
-    default:
-      fn = sys_scope ? kernel_ptr<kBFloat16, true>() : kernel_ptr<kBFloat16, false>();
-      break;
+  if (sgd) {
+    fn = sys_scope ? kernel_ptr<kFloat32, true, true>(threads) : kernel_ptr<kFloat32, false, true>(threads);
+  } else {
+    switch (dtype) {
+      case kInt32:
+        fn = sys_scope ? kernel_ptr<kInt32, true, false>(threads) : kernel_ptr<kInt32, false, false>(threads);
+        break;
+      case kFloat32:
+        fn = sys_scope ? kernel_ptr<kFloat32, true, false>(threads) : kernel_ptr<kFloat32, false, false>(threads);
+        break;
+      default:
+        fn = sys_scope ? kernel_ptr<kBFloat16, true, false>(threads)
+                       : kernel_ptr<kBFloat16, false, false>(threads);
+        break;
+    }
   }
   return static_cast<int>(cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks, fn, threads, 0));
 }

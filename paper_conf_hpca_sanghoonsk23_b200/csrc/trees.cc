@@ -5,7 +5,8 @@
 // nodes and leaves" (fn4 P:L153).  Reading R1: binary tree
 // rooted at rank 0 with one child; rank r (lowest set bit b) has children
 // r - b/2 and r + b/2, the right offset halved until it is < P.  Tree 1 renames
-// every rank v of tree 0 to P-1-v (even P) or (v+1) mod P (odd P).
+// every rank v of tree 0 to P-1-v (even P) or (v+1) mod P (odd P).  The ROTATED
+// set renames tree 0 by v -> (v + t) mod P for t = 0..P-1.
 //
 // This builder works top-down from the children rule; the oracle builds the same
 // tree bottom-up from a parent rule, and tests/test_abi_host.py checks that the
@@ -46,11 +47,16 @@ void build_tree0(int P, Tree *t) {
   }
 }
 
-int rename(int P, int v) { return (P % 2 == 0) ? (P - 1 - v) : ((v + 1) % P); }
+int rename(int P, int kind, int which, int v) {
+  if (kind == 2) return (v + which) % P;
+  return (P % 2 == 0) ? (P - 1 - v) : ((v + 1) % P);
+}
 
 }  // namespace
 
-void build_tree(int P, int which, Tree *out) {
+int num_trees(int P, int kind) { return kind == 2 ? (P > 1 ? P : 1) : kind == 1 ? 2 : 1; }
+
+void build_tree(int P, int kind, int which, Tree *out) {
   Tree t0;
   build_tree0(P, &t0);
   if (which == 0) {
@@ -58,11 +64,11 @@ void build_tree(int P, int which, Tree *out) {
     return;
   }
   out->P = P;
-  out->root = rename(P, t0.root);
+  out->root = rename(P, kind, which, t0.root);
   for (int v = 0; v < P; ++v) out->nchild[v] = 0;
   for (int v = 0; v < P; ++v) {
-    const int nv = rename(P, v);
-    out->parent[nv] = t0.parent[v] < 0 ? -1 : rename(P, t0.parent[v]);
+    const int nv = rename(P, kind, which, v);
+    out->parent[nv] = t0.parent[v] < 0 ? -1 : rename(P, kind, which, t0.parent[v]);
   }
   // children in ascending rank (the combine order, R2)
   for (int c = 0; c < P; ++c) {

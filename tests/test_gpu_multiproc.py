@@ -84,6 +84,7 @@ def _run(world, kind, dtype, count, chunk):
 
 
 @pytest.mark.parametrize("world,kind,dtype", [(2, "single", "float32"),
+                                              (4, "rotated", "float32"),
                                               (3, "double", "bfloat16"),
                                               (4, "double", "float32"),
                                               (4, "single", "int32")])

@@ -285,3 +285,125 @@ def test_landing_trace_in_order_and_c1_turnaround(comm):
     turn_b, total_b = res[False]
     turn_c, total_c = res[True]
     assert turn_c * 4 < turn_b, res
+
+
+# ---- rotated multi-tree set (reading R17) ---------------------------
+@pytest.mark.parametrize("P", [2, 3, 4, 8])
+@pytest.mark.parametrize("dtype", ["int32", "float32", "bfloat16"])
+@pytest.mark.parametrize("overlap", [True, False])
+@pytest.mark.parametrize("transport", ["pull", "push"])
+def test_parity_rotated(comm, P, dtype, overlap, transport):
+    """P trees, chunk c on tree c mod P: bit-exact vs the oracle definition, with
+    several chunks per tree and a ragged tail."""
+    chunk = 4096
+    comm(P, "rotated", chunk, channels=2, overlap=overlap, transport=transport)
+    E = chunk // arith.ELEM_SIZE[dtype]
+    count = (2 * P + 3) * E + 13
+    xs, outs = _run(P, "rotated", dtype, count, chunk)
+    ref = oar.reference(xs, "rotated", chunk, dtype)[0]
+    for r in range(P):
+        assert np.array_equal(outs[r], ref), f"rank {r}"
+
+
+def test_full_size_resnet50_rotated(comm):
+    """ResNet-50 gradient set over the rotated set at P = 8 (auto channels): sampled
+    chunks of every tree bit-exact vs the oracle, every rank identical."""
+    P, chunk = 8, 256 << 10
+    comm(P, "rotated", chunk)
+    count, ends, ts = _full_size(P, "rotated", "float32", "resnet50", chunk)
+    K = partition.num_chunks(count, chunk, 4)
+    for c in sorted({0, 1, 2, 3, 4, 5, 6, 7, K - 2, K - 1, 200}):
+        lo, hi, want = oracle_chunk(P, "rotated", chunk, "float32", count, c, layer_ends=ends)
+        for r in (0, 5):
+            assert np.array_equal(to_numpy(ts[r][lo:hi], "float32"), want), (c, r)
+    for r in range(1, P):
+        assert torch.equal(ts[r], ts[0])
+
+
+def test_gradient_queue_gates_rotated(comm):
+    """a9 with P trees: layer l needs #{c < LCT[l] : c mod P = t} chunks of tree t."""
+    P, chunk = 8, 64 << 10
+    comm(P, "rotated", chunk, channels=2)
+    ends = workloads.layer_ends("resnet50")
+    count = ends[-1]
+    ts = device_inputs(P, count, "float32", layer_ends=ends)
+    ccube.gradq_set_layers(ends)
+    comm_stream, comp = torch.cuda.Stream(), torch.cuda.Stream()
+    comm_stream.wait_stream(torch.cuda.current_stream())
+    comp.wait_stream(torch.cuda.current_stream())
+    snaps = {}
+    rank = 3
+    with torch.cuda.stream(comm_stream):
+        ccube.allreduce_tree_local(ts, stream=comm_stream)
+    with torch.cuda.stream(comp):
+        starts = [0] + ends[:-1]
+        for l in range(len(ends)):
+            ccube.gradq_wait_local(rank, l, stream=comp)
+            snaps[l] = ts[rank][starts[l]:ends[l]].clone()
+    torch.cuda.synchronize()
+    for l in range(len(ends)):
+        assert torch.equal(snaps[l], ts[rank][starts[l]:ends[l]]), f"layer {l} read before landing"
+
+
+# ---- fused SGD update at dequeue (reading R18) ----------------------
+@pytest.mark.parametrize("P", [2, 4, 8])
+@pytest.mark.parametrize("kind", ["single", "double", "rotated"])
+@pytest.mark.parametrize("overlap", [True, False])
+def test_fused_sgd_parity(comm, P, kind, overlap):
+    """Every rank's weights become oracle.gradq.sgd_update(w, final, alpha) bit for
+    bit (root: in its reduce; interior: in its broadcast; leaf: UPDATE task), and
+    the gradients are still the oracle's fixed-order sum.  Ragged fp32 tail."""
+    from oracle import gradq as ogq
+    chunk = 4096
+    comm(P, kind, chunk, channels=2, overlap=overlap)
+    E = chunk // 4
+    count = 7 * E + 13
+    ws0 = [inputs.gradients(r + 100, count, "float32") for r in range(P)]
+    ws = [to_torch(w, "float32").cuda() for w in ws0]
+    alpha = 0.013
+    ccube.gradq_set_sgd(ws, alpha)
+    xs, outs = _run(P, kind, "float32", count, chunk)
+    ref = oar.reference(xs, kind, chunk, "float32")[0]
+    for r in range(P):
+        assert np.array_equal(outs[r], ref), f"grads rank {r}"
+        want = ogq.sgd_update(ws0[r], ref, alpha)
+        assert np.array_equal(to_numpy(ws[r], "float32"), want), f"weights rank {r}"
+    ccube.gradq_set_sgd(None)
+
+
+def test_fused_sgd_gate_waits_for_weights(comm):
+    """With the fused update the gate opens once the layer's weights are updated."""
+    P, chunk, rank = 8, 64 << 10, 5
+    comm(P, "double", chunk, channels=2)
+    ends = workloads.layer_ends("resnet50")
+    count = ends[-1]
+    ts = device_inputs(P, count, "float32", layer_ends=ends)
+    ws = device_inputs(P, count, "float32", seed=99)
+    ccube.gradq_set_layers(ends)
+    ccube.gradq_set_sgd(ws, 0.01)
+    comm_stream, comp = torch.cuda.Stream(), torch.cuda.Stream()
+    comm_stream.wait_stream(torch.cuda.current_stream())
+    comp.wait_stream(torch.cuda.current_stream())
+    snaps = {}
+    with torch.cuda.stream(comm_stream):
+        ccube.allreduce_tree_local(ts, stream=comm_stream)
+    with torch.cuda.stream(comp):
+        starts = [0] + ends[:-1]
+        for l in range(len(ends)):
+            ccube.gradq_wait_local(rank, l, stream=comp)
+            snaps[l] = ws[rank][starts[l]:ends[l]].clone()
+    torch.cuda.synchronize()
+    for l in range(len(ends)):
+        assert torch.equal(snaps[l], ws[rank][starts[l]:ends[l]]), f"layer {l} weights early"
+    ccube.gradq_set_sgd(None)
+
+
+def test_fused_sgd_rejects_non_fp32(comm):
+    comm(4, "single", 4096)
+    ws = [torch.zeros(4096, device="cuda") for _ in range(4)]
+    ccube.gradq_set_sgd(ws, 0.1)
+    ts = [torch.zeros(2048, dtype=torch.bfloat16, device="cuda") for _ in range(4)]
+    with pytest.raises(ccube.CCubeError) as e:
+        ccube.allreduce_tree_local(ts)
+    assert e.value.code == ccube.ERR_INVALID_ARG
+    ccube.gradq_set_sgd(None)

@@ -122,3 +122,82 @@ def test_chained_training_equals_unchained(kind):
         finals[chained] = [p.detach().cpu() for p in m.parameters()]
     for a, b in zip(finals[False], finals[True]):
         assert torch.equal(a, b)
+
+
+def test_views_keep_channels_last_strides():
+    m = torchvision.models.resnet50(weights=None).to(memory_format=torch.channels_last)
+    strides = {n: p.stride() for n, p in m.named_parameters()}
+    gq = attach_gradient_queue(m)
+    for n, p in m.named_parameters():   # strides of size-1 dims carry no layout
+        assert p.grad.shape == p.shape
+        assert [s for s, k in zip(p.grad.stride(), p.shape) if k > 1] == \
+            [s for s, k in zip(strides[n], p.shape) if k > 1]
+    gq.remove()
+
+
+def test_fused_mode_moves_weights_into_flat_buffer():
+    m = _tiny()
+    before = [p.detach().clone() for p in m.parameters()]
+    gq = attach_gradient_queue(m, lr=0.1, world_size=2, fused_sgd=True)
+    off = 0
+    for b, p in zip(before, m.parameters()):
+        assert torch.equal(p.detach(), b)
+        assert p.data_ptr() == gq.flat_w[off:].data_ptr()
+        off += p.numel()
+    # the pre-hook no longer updates (the AllReduce kernel does)
+    x = torch.randn(2, 3, 8, 8)
+    m(x).sum().backward()
+    gq.update = True
+    with torch.no_grad():
+        m(x)
+    for b, p in zip(before, m.parameters()):
+        assert torch.equal(p.detach(), b)
+    gq.remove()
+
+
+@pytest.mark.gpu
+def test_fused_chained_training_equals_fused_unchained():
+    """f2 + C2: with the update fused into the AllReduce, chaining still changes
+    timing only."""
+    from paper_conf_hpca_sanghoonsk23_b200 import ccube
+    torch.backends.cudnn.deterministic = True
+    torch.backends.cudnn.benchmark = False
+    P, rr = 4, 2
+    finals = {}
+    for chained in (False, True):
+        m = _tiny().cuda()
+        gq = attach_gradient_queue(m, lr=0.1, world_size=P, local_rank=rr, fused_sgd=True)
+        others = [torch.zeros_like(gq.flat) for _ in range(P - 1)]
+        bufs = others[:rr] + [gq.flat] + others[rr:]
+        ow = [gq.flat_w.clone() for _ in range(P - 1)]
+        wts = ow[:rr] + [gq.flat_w] + ow[rr:]
+        comp, comm = torch.cuda.Stream(), torch.cuda.Stream()
+        ccube.init_loopback(P, "double", 256)
+        try:
+            ccube.set_channels(2)
+            gq.set_layers(weights=wts)
+            gq.chained = chained
+            g = torch.Generator().manual_seed(4)
+            for it in range(3):
+                x = torch.randn(16, 3, 8, 8, generator=g).cuda()
+                with torch.cuda.stream(comp):
+                    loss = m(x).square().mean()
+                    comp.wait_stream(comm)
+                    gq.zero_()
+                    loss.backward()
+                    for r, o in enumerate(others):
+                        o.copy_(gq.flat * (r + 2))
+                comm.wait_stream(comp)
+                ccube.allreduce_tree_local(bufs, stream=comm)
+                if not chained:
+                    comp.wait_stream(comm)
+            with torch.cuda.stream(comp), torch.no_grad():
+                m(torch.zeros(1, 3, 8, 8, device="cuda"))
+            torch.cuda.synchronize()
+        finally:
+            gq.remove()
+            ccube.finalize()
+        finals[chained] = [p.detach().cpu() for p in m.parameters()]
+        assert not torch.equal(finals[chained][0], _tiny().state_dict()["0.weight"])
+    for a, b in zip(finals[False], finals[True]):
+        assert torch.equal(a, b)

@@ -1,5 +1,6 @@
 """Pins for oracle.gradq: Fig 8 Layer-Chunk Table, Fig 11 semaphore semantics, gates."""
 
+import numpy as np
 import pytest
 
 from oracle import gradq, schedule, trees
@@ -86,3 +87,23 @@ def test_forward_timeline_model():
     assert chained == [5, 8, 10, 11, 16]
     assert unchained == [19, 22, 24, 25, 26]
     assert chained[-1] <= unchained[-1]
+
+
+def test_sgd_update_closed_forms():
+    """R18: w - alpha * g elementwise; exact cases."""
+    w = np.array([1.0, -2.0, 3.5, 0.0], dtype=np.float32)
+    g = np.array([2.0, 4.0, -1.0, 0.0], dtype=np.float32)
+    assert np.array_equal(gradq.sgd_update(w, g, 0.5), np.array([0.0, -4.0, 4.0, 0.0], np.float32))
+    assert np.array_equal(gradq.sgd_update(w, g, 0.0), w)
+    assert gradq.sgd_update(w, g, 0.5).dtype == np.float32
+
+
+def test_sgd_update_rounds_twice_no_fma(golden):
+    """R18 pin: the product is rounded before the subtraction (an FMA differs)."""
+    gl = golden("order_pins.txt")
+    w, g, a = (float(v) for v in gl["sgd_no_fma_pin_w_g_alpha"])
+    got = gradq.sgd_update(np.array([w], np.float32), np.array([g], np.float32), a)[0]
+    assert got == float(gl["sgd_no_fma_pin_result"][0])
+    exact = w - a * g          # python floats are binary64: exact here
+    assert exact == float(gl["sgd_fma_result"][0])
+    assert np.float32(exact) != got
