@@ -72,6 +72,8 @@ struct TreeParams {
   int child_interior[kMaxChildren]; // child has children: its buffer is re-read (DOWN)
   char *w;                          // own fp32 weights (fused SGD, f2), same layout as buf
   uint64_t *upd;                    // own "weights updated" counter (channel 0)
+  uint32_t pf_mask;                 // bit q: up_src[q] is a raw input (own buf, a pulled
+                                    // leaf's buf), readable from the start: L2 prefetch
 };
 
 // UPDATE: a leaf's fused-SGD task (f2) — waits for its chunks to land, then
@@ -105,6 +107,9 @@ struct LaunchArgs {
   int l2_hints;               // 1 = per-stream L2 eviction priorities (keep re-read data)
   int sgd;                    // 1 = fused SGD update at landing (fp32 only)
   float sgd_alpha;            // w <- w - sgd_alpha * g
+  int tma;                    // datapath: 0 = register-staged LSU, 1 = TMA bulk-load ring
+  int prefetch;               // UP tasks prefetch raw inputs this many chunks ahead (0 = off)
+  int elem_size;              // bytes per element (2 or 4)
 };
 
 // Kernel launcher (tree_allreduce.cu).  Returns a cudaError_t as int.
@@ -113,6 +118,7 @@ int launch_tree_allreduce(const LaunchArgs &args, int dtype, bool sys_scope, int
 constexpr int kMaxGateCounters = 128;
 int launch_gate(const uint64_t *const *counters, const uint64_t *targets, int n, int *err,
                 uint64_t timeout_ns, bool sys_scope, void *stream);
-int query_max_blocks_per_sm(int dtype, bool sys_scope, bool sgd, int threads, int *blocks);
+int query_max_blocks_per_sm(int dtype, bool sys_scope, bool sgd, int threads, int tma,
+                            int *blocks);
 
 }  // namespace ccube

@@ -166,6 +166,8 @@ struct Comm {
   int last_channels = 0;
   int last_ctas = 0;
   int l2_hints = 1;
+  int datapath = CCUBE_DATAPATH_LSU;  // CCUBE_DATAPATH env / ccube_set_datapath
+  int prefetch = 0;                   // CCUBE_PREFETCH env: chunks of L2 prefetch ahead
   bool sgd = false;                 // fused SGD update (f2)
   float sgd_alpha = 0.0f;
   size_t sgd_bytes = 0;
@@ -182,7 +184,7 @@ struct Comm {
   bool sys_scope = false;
   uint64_t timeout_ns = 10000ull * 1000000ull;
   int sm_count = 0;
-  std::map<std::pair<int, int>, int> max_blocks;  // (dtype, threads)
+  std::map<std::pair<int, int>, int> max_blocks;  // (dtype*2+sgd + 8*datapath, threads)
   uint64_t *trace = nullptr;
   size_t trace_kmax = 0;
   bool use_memop = true;
@@ -301,6 +303,7 @@ ccube_result_t build_params(Registration *R) {
       memset(&p, 0, sizeof p);
       p.buf = R->bufs[i];
       p.up_src[0] = R->bufs[i];
+      p.pf_mask = 1u;  // my own input
       p.nchild = tr.nchild[r];
       p.is_root = tr.parent[r] < 0;
       p.self_local = i;
@@ -340,6 +343,7 @@ ccube_result_t build_params(Registration *R) {
         p.child_interior[s] = tr.nchild[c] > 0;
         if (edge_is_pull(c, r)) {
           p.up_src[1 + s] = R->world_buf[c];
+          if (tr.nchild[c] == 0) p.pf_mask |= 2u << s;  // a pulled leaf: its raw input
         } else {
           if (!R->recv[i]) return fail(CCUBE_ERR_BOOTSTRAP, "receive plane missing");
           p.up_src[1 + s] = R->recv[i] + static_cast<size_t>(s) * R->plane;
@@ -510,11 +514,13 @@ ccube_result_t allreduce_impl(void *const *bufs, size_t count, ccube_dtype_t dty
 
   // all CTAs spin on each other: they must be co-resident
   const int cta_threads = g.threads + 32;  // data warps + the control warp
-  auto key = std::make_pair((int)dtype * 2 + (g.sgd ? 1 : 0), cta_threads);
+  // the TMA datapath needs a producer and at least one consumer data warp
+  const int tma = g.datapath == CCUBE_DATAPATH_TMA && g.threads >= 64 ? 1 : 0;
+  auto key = std::make_pair((int)dtype * 2 + (g.sgd ? 1 : 0) + 8 * tma, cta_threads);
   if (!g.max_blocks.count(key)) {
     int b = 0;
     const int rc =
-        query_max_blocks_per_sm(dtype, g.sys_scope, g.sgd, cta_threads, &b);
+        query_max_blocks_per_sm(dtype, g.sys_scope, g.sgd, cta_threads, tma, &b);
     if (rc != cudaSuccess)
       return fail(CCUBE_ERR_CUDA, "occupancy query failed: %s",
                   cudaGetErrorString(static_cast<cudaError_t>(rc)));
@@ -525,11 +531,14 @@ ccube_result_t allreduce_impl(void *const *bufs, size_t count, ccube_dtype_t dty
   if (J == 0) {  // auto: the most channels whose CTAs all fit at once ...
     J = 1;
     while (J < CCUBE_MAX_CHANNELS && count_tasks(J + 1, g.overlap) <= cap) ++J;
-    // ... but at least two 2 KB units per channel and chunk: a small buffer gets
-    // few channels, so few CTAs take part in the handshakes (latency)
+    // ... but at least two 2 KB units per channel and chunk while the buffer is a
+    // few chunks long: a small buffer gets few channels, so few CTAs take part in
+    // the handshakes (latency).  A long buffer is bandwidth-bound, so it may use
+    // one unit per channel (P=2 at 256 KiB chunks: 128 channels instead of 64).
     const uint64_t first = bytes < g.chunk_bytes ? bytes : g.chunk_bytes;
     const uint64_t units = (first + 2047) / 2048;
-    const int jmax = units / 2 > 1 ? static_cast<int>(units / 2) : 1;
+    const uint64_t per = bytes >= 16 * g.chunk_bytes ? 1 : 2;
+    const int jmax = units / per > 1 ? static_cast<int>(units / per) : 1;
     if (J > jmax) J = jmax;
   }
 
@@ -550,6 +559,9 @@ ccube_result_t allreduce_impl(void *const *bufs, size_t count, ccube_dtype_t dty
   a.l2_hints = g.l2_hints;
   a.sgd = g.sgd ? 1 : 0;
   a.sgd_alpha = g.sgd_alpha;
+  a.tma = tma;
+  a.prefetch = g.prefetch;
+  a.elem_size = static_cast<int>(es);
   a.params = R->d_params;
 
   TaskTable *tt = nullptr;
@@ -719,6 +731,11 @@ ccube_result_t ccube_init(const ccube_world_t *world, ccube_tree_kind_t tree_kin
   g.transport = transport;
   g.overlap = 1;
   g.l2_hints = env_int("CCUBE_L2_HINTS", 1);
+  g.datapath = env_int("CCUBE_DATAPATH", CCUBE_DATAPATH_LSU) == CCUBE_DATAPATH_TMA
+                   ? CCUBE_DATAPATH_TMA
+                   : CCUBE_DATAPATH_LSU;
+  g.prefetch = env_int("CCUBE_PREFETCH", 0);
+  if (g.prefetch < 0) g.prefetch = 0;
   g.sys_scope = g.nproc > 1;
   g.timeout_ns = static_cast<uint64_t>(env_int("CCUBE_WATCHDOG_MS", 10000)) * 1000000ull;
   g.use_memop = env_int("CCUBE_GATE_KERNEL", 0) == 0;
@@ -932,6 +949,24 @@ ccube_result_t ccube_set_threads(int threads) {
   return CCUBE_SUCCESS;
 }
 
+ccube_result_t ccube_set_datapath(int datapath) {
+  std::lock_guard<std::mutex> lk(g_mu);
+  if (!g.init) return fail(CCUBE_ERR_NOT_INITIALIZED, "ccube_init has not been called");
+  if (datapath != CCUBE_DATAPATH_LSU && datapath != CCUBE_DATAPATH_TMA)
+    return fail(CCUBE_ERR_INVALID_ARG, "datapath %d out of range", datapath);
+  g.datapath = datapath;
+  return CCUBE_SUCCESS;
+}
+
+ccube_result_t ccube_set_prefetch(int chunks) {
+  std::lock_guard<std::mutex> lk(g_mu);
+  if (!g.init) return fail(CCUBE_ERR_NOT_INITIALIZED, "ccube_init has not been called");
+  if (chunks < 0 || chunks > 1024)
+    return fail(CCUBE_ERR_INVALID_ARG, "prefetch %d out of range [0, 1024]", chunks);
+  g.prefetch = chunks;
+  return CCUBE_SUCCESS;
+}
+
 ccube_result_t ccube_set_transport(int mode) {
   std::lock_guard<std::mutex> lk(g_mu);
   if (!g.init) return fail(CCUBE_ERR_NOT_INITIALIZED, "ccube_init has not been called");
@@ -997,6 +1032,8 @@ ccube_result_t ccube_get_info(ccube_info_t *info) {
   info->epoch_base[1] = g.base[1];
   info->last_channels = g.last_channels;
   info->last_ctas = g.last_ctas;
+  info->datapath = g.datapath;
+  info->prefetch = g.prefetch;
   return CCUBE_SUCCESS;
 }
 

@@ -431,10 +431,26 @@ __device__ __forceinline__ void st_hint(char *ptr, const uint4 &v, uint64_t pol)
                : "memory");
 }
 
+// TMA datapath (kDatapathTma): a shared-memory ring of stages, each holding one block
+// (<= kTmaSeg bytes) of every source; see tma_produce / tma_consume below.
+constexpr uint32_t kTmaRing = 96u * 1024u;  // two CTAs per SM: 2 x 96 KB of the 228 KB
+constexpr uint32_t kTmaSeg = 8192;          // bytes per source per stage (at most)
+constexpr int kTmaMaxStages = 12;           // one source: 12 x 8 KB
+constexpr uint32_t kTmaAbort = 0xffffffffu;
+
+struct TmaDesc {
+  uint64_t off;    // byte offset of the block in the buffers
+  uint32_t len;    // bytes (kTmaAbort = stop)
+  uint32_t kdone;  // after this block every chunk < kdone is finished (tree-local)
+};
+
 struct Shared {
   uint64_t ready;                // chunks whose inputs are available (control -> data)
   uint64_t done[kMaxDataWarps];  // chunks finished by data warp w (data -> control)
   int abort;
+  uint64_t full[kTmaMaxStages];  // TMA: stage loaded (complete_tx)
+  uint64_t empty[kTmaMaxStages]; // TMA: stage consumed by every consumer warp
+  TmaDesc desc[kTmaMaxStages];
 };
 
 // CTA-scope release/acquire on shared memory (control <-> data warps)
@@ -536,6 +552,35 @@ __device__ __forceinline__ void combine_scalar(const char *const *src, int nin, 
 // each data warp streams its blocks (BlockIter) and reports, through a per-warp
 // "done" counter, the chunk of its next block; the control warp publishes the
 // minimum over the warps downstream.
+// L2 prefetch of an UP task's raw inputs (own buffer, pulled leaves' buffers): they
+// sit in DRAM from the start, so the control warp keeps `a.prefetch` chunks of this
+// channel's slices in flight ahead of the data warps with bulk L2 prefetches (no
+// registers, no shared memory).  The data warps' loads then hit L2: the DRAM latency
+// leaves the critical path of the DRAM-heavy tasks.  Prefetching is only a hint —
+// L2 is the point of coherence, so a line prefetched early is still updated by any
+// later write.
+struct Prefetcher {
+  Geo g;
+  uint32_t k, c;   // next chunk to prefetch, k mod J
+  uint64_t c0;     // its byte offset
+  const char *src; // this lane's source (nullptr = none)
+};
+
+__device__ __forceinline__ void prefetch_l2(const void *ptr, uint32_t bytes) {
+  asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(ptr), "r"(bytes) : "memory");
+}
+
+__device__ __forceinline__ void prefetch_until(Prefetcher &pf, uint32_t upto) {
+  while (pf.k < pf.g.K && pf.k < upto) {
+    const Slice sl = slice_at(pf.g, pf.c, pf.c0);
+    const uint32_t len = sl.len & ~15u;
+    if (pf.src && len) prefetch_l2(pf.src + sl.off, len);
+    ++pf.k;
+    pf.c = pf.c + 1 == pf.g.J ? 0 : pf.c + 1;
+    pf.c0 += pf.g.stride;
+  }
+}
+
 template <bool SYS>
 __device__ void control_warp(const LaunchArgs &a, const TreeParams &p, int role, int t, int j,
                              int W, Shared &sh) {
@@ -543,6 +588,17 @@ __device__ void control_warp(const LaunchArgs &a, const TreeParams &p, int role,
   const uint32_t K = a.K[t];
   const uint64_t base = a.base[t];
   const int stride = j * kFlagStrideU64;
+  const bool do_pf = role == kRoleUp && a.prefetch > 0 && lane <= p.nchild &&
+                     ((p.pf_mask >> lane) & 1u);
+  Prefetcher pf;
+  if (do_pf) {
+    pf.g = a.elem_size == 2 ? make_geo<2>(a, t, j) : make_geo<4>(a, t, j);
+    pf.k = 0;
+    pf.c = 0;
+    pf.c0 = pf.g.first;
+    pf.src = p.up_src[lane];
+    prefetch_until(pf, static_cast<uint32_t>(a.prefetch));
+  }
   const uint64_t *up = nullptr;
   if (role == kRoleUp) {
     if (lane < p.nchild) up = p.head_in[lane] + stride;
@@ -577,6 +633,7 @@ __device__ void control_warp(const LaunchArgs &a, const TreeParams &p, int role,
       if (lane == 0) publish<SYS>(a, p, role, t, j, pub, static_cast<uint32_t>(d), base);
       pub = static_cast<uint32_t>(d);
       moved = true;
+      if (do_pf) prefetch_until(pf, pub + static_cast<uint32_t>(a.prefetch));
     }
     if (moved) {
       watch_reset(wd);
@@ -707,6 +764,210 @@ __device__ __forceinline__ void lsu_nout(const LaunchArgs &a, const Endpoints &e
   }
 }
 
+// ---- TMA datapath (kDatapathTma) ---------------------------------------------------
+// Data warp 0 is a producer: one lane walks this channel's blocks in chunk order (the
+// same BlockIter as the LSU path, with kTmaSeg blocks and W = 1), waits for the
+// control warp's "ready", and streams each block of every source into a ring stage
+// with cp.async.bulk (mbarrier complete_tx).  Data warps 1..W-1 consume every stage:
+// the fixed-order combine from shared memory, 128-bit stores to the destinations,
+// then an arrive on the stage's "empty" barrier.  All sources are local (own buffer,
+// own receive planes, or a same-GPU child's buffer on a PULL edge), so the bulk
+// loads never cross NVLink; stores still go out as generic 128-bit stores, so the
+// release chain to the control warp is the LSU path's.  The ring holds up to
+// kTmaRing bytes in flight per CTA without registers: what the DRAM-heavy tasks
+// lack in the register-staged path (tools/membench2.cu).
+__device__ __forceinline__ void mbar_init(uint64_t *m, uint32_t n) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(m)), "r"(n) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t *m, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(m)),
+               "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t *m) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(m)) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t *m, uint32_t parity) {
+  asm volatile(
+      "{\n .reg .pred p;\n WAIT_%=:\n"
+      " mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+      " @!p bra WAIT_%=;\n}\n" ::"r"(smem_u32(m)),
+      "r"(parity)
+      : "memory");
+}
+__device__ __forceinline__ void bulk_load(void *smem, const void *gptr, uint32_t bytes,
+                                          uint64_t *m, uint64_t pol) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint"
+      " [%0], [%1], %2, [%3], %4;" ::"r"(smem_u32(smem)),
+      "l"(gptr), "r"(bytes), "r"(smem_u32(m)), "l"(pol)
+      : "memory");
+}
+
+__device__ __forceinline__ int tma_nsrc(const Endpoints &e) { return e.nin + (e.sgd ? 1 : 0); }
+__device__ __forceinline__ int tma_stages(int nsrc) {
+  const int s = static_cast<int>(kTmaRing / (nsrc * kTmaSeg));
+  return s < kTmaMaxStages ? s : kTmaMaxStages;
+}
+
+__device__ void tma_produce(const LaunchArgs &a, const Endpoints &e, int t, int j, Shared &sh,
+                            char *ring) {
+  const int ES = a.elem_size;
+  const Geo g = ES == 2 ? make_geo<2>(a, t, j) : make_geo<4>(a, t, j);
+  const int nsrc = tma_nsrc(e);
+  const int S = tma_stages(nsrc);
+  const char *src[kMaxIn + 1];
+  for (int q = 0; q < e.nin; ++q) src[q] = e.src[q];
+  if (e.sgd) src[e.nin] = e.w;
+  const L2Pol pol = make_pol(a.l2_hints);
+  uint64_t ready = 0;
+  uint32_t i = 0;
+  BlockIter it = iter_begin<kTmaSeg>(g, 0);
+  bool aborted = false;
+  while (it.k < g.K || i == 0) {  // an empty walk still sends one "all done" stage
+    const uint32_t k = it.k;
+    if (k < g.K && k >= ready) {
+      uint64_t r;
+      while ((r = ld_acquire_cta(&sh.ready)) <= k && !*reinterpret_cast<volatile int *>(&sh.abort))
+        __nanosleep(64);
+      if (r <= k) {
+        aborted = true;
+        break;
+      }
+      ready = r;
+      // the upstream data was acquired through the generic proxy; the bulk loads
+      // below read it through the async proxy
+      asm volatile("fence.proxy.async.global;" ::: "memory");
+    }
+    const int s = static_cast<int>(i % S);
+    if (i >= static_cast<uint32_t>(S)) mbar_wait(&sh.empty[s], ((i / S) - 1) & 1);
+    uint64_t off = 0;
+    uint32_t len = 0;
+    if (k < g.K) {
+      const uint32_t b0 = it.s * kTmaSeg;
+      off = it.sl.off + b0;
+      len = min(kTmaSeg, it.sl.len - b0);
+      it.s += 1;
+      iter_settle<kTmaSeg>(g, it);
+    }
+    sh.desc[s].off = off;
+    sh.desc[s].len = len;
+    sh.desc[s].kdone = it.k;
+    const uint32_t vlen = len & ~15u;
+    if (vlen) {
+      mbar_expect_tx(&sh.full[s], vlen * nsrc);
+      for (int q = 0; q < nsrc; ++q)
+        bulk_load(ring + (s * nsrc + q) * kTmaSeg, src[q] + off, vlen, &sh.full[s], pol.first);
+    } else {
+      mbar_arrive(&sh.full[s]);
+    }
+    ++i;
+  }
+  if (aborted) {  // wake every consumer with a stop stage
+    const int s = static_cast<int>(i % S);
+    if (i >= static_cast<uint32_t>(S)) mbar_wait(&sh.empty[s], ((i / S) - 1) & 1);
+    sh.desc[s].len = kTmaAbort;
+    mbar_arrive(&sh.full[s]);
+  }
+}
+
+template <int DT, int NIN, int NOUT, bool SGD>
+__device__ void tma_consume(const LaunchArgs &a, const Endpoints &e, int t, int w, int cw,
+                            int CW, Shared &sh, const char *ring) {
+  constexpr int NSRC = NIN + (SGD ? 1 : 0);
+  const int lane = threadIdx.x & 31;
+  const int S = tma_stages(NSRC);
+  const uint32_t K = a.K[t];
+  const L2Pol pol = make_pol(a.l2_hints);
+  const float alpha = a.sgd_alpha;
+  uint64_t dpol[NOUT > 0 ? NOUT : 1];
+#pragma unroll
+  for (int q = 0; q < NOUT; ++q) dpol[q] = (e.keep >> q) & 1u ? pol.last : pol.first;
+  uint32_t done_reported = 0;
+  for (uint32_t i = 0;; ++i) {
+    const int s = static_cast<int>(i % S);
+    mbar_wait(&sh.full[s], (i / S) & 1);
+    const TmaDesc d = sh.desc[s];
+    if (d.len == kTmaAbort) return;
+    const uint32_t nvec = d.len / 16;
+    const uint4 *st = reinterpret_cast<const uint4 *>(ring + s * NSRC * kTmaSeg);
+    constexpr uint32_t kSegVec = kTmaSeg / 16;
+#pragma unroll 2
+    for (uint32_t v = cw * 32 + lane; v < nvec; v += CW * 32) {
+      uint4 x[NIN];
+#pragma unroll
+      for (int q = 0; q < NIN; ++q) x[q] = st[q * kSegVec + v];
+      const uint4 r = Combine<DT>::template vec<NIN>(x);
+      const uint64_t o = d.off + 16ull * v;
+#pragma unroll
+      for (int q = 0; q < NOUT; ++q) st_hint(e.dst[q] + o, r, dpol[q]);
+      if constexpr (SGD) st_hint(e.w + o, sgd4(st[NIN * kSegVec + v], r, alpha), pol.first);
+    }
+    if ((d.len & 15u) && cw == 0) {  // ragged end of the buffer (< 16 bytes)
+      const uint64_t o = d.off + (d.len & ~15u);
+      if (NOUT > 0) combine_scalar<DT>(e.src, NIN, e.dst, NOUT, o, d.len & 15u);
+      if constexpr (SGD) {
+        __syncwarp();
+        for (uint32_t x4 = lane; x4 < (d.len & 15u) / 4; x4 += 32) {
+          float *wp = reinterpret_cast<float *>(e.w + o) + x4;
+          *wp = sgd1(*wp, reinterpret_cast<const float *>(e.gfinal + o)[x4], alpha);
+        }
+      }
+    }
+    __syncwarp();  // every lane is done with the stage and its stores precede the release
+    if (lane == 0) {
+      mbar_arrive(&sh.empty[s]);
+      if (d.kdone > done_reported) st_release_cta(&sh.done[w], d.kdone);
+    }
+    done_reported = d.kdone > done_reported ? d.kdone : done_reported;
+    if (done_reported >= K) return;
+  }
+}
+
+template <int DT, int NIN, bool SGD>
+__device__ __forceinline__ void tma_nout(const LaunchArgs &a, const Endpoints &e, int t, int w,
+                                         int cw, int CW, Shared &sh, const char *ring) {
+  if constexpr (SGD && DT == kFloat32 && NIN <= 2) {
+    if (e.sgd) {
+      switch (e.nout) {
+        case 0: tma_consume<DT, NIN, 0, true>(a, e, t, w, cw, CW, sh, ring); return;
+        case 1: tma_consume<DT, NIN, 1, true>(a, e, t, w, cw, CW, sh, ring); return;
+        default: tma_consume<DT, NIN, 2, true>(a, e, t, w, cw, CW, sh, ring); return;
+      }
+    }
+  }
+  switch (e.nout) {
+    case 1: tma_consume<DT, NIN, 1, false>(a, e, t, w, cw, CW, sh, ring); break;
+    case 2: tma_consume<DT, NIN, 2, false>(a, e, t, w, cw, CW, sh, ring); break;
+    default: tma_consume<DT, NIN, 3, false>(a, e, t, w, cw, CW, sh, ring); break;
+  }
+}
+
+// Data warp w of W on the TMA datapath: w == 0 produces (lane 0), the others consume.
+template <int DT, bool SGD>
+__device__ void tma_data_warp(const LaunchArgs &a, const TreeParams &p, int role, int t, int j,
+                              int w, int W, Shared &sh, char *ring) {
+  Endpoints e = endpoints(a, p, role);
+  if (!SGD) e.sgd = false;
+  const int lane = threadIdx.x & 31;
+  if (e.nout == 0 && !e.sgd) {  // nothing to write (cannot happen for scheduled tasks)
+    if (lane == 0) st_release_cta(&sh.done[w], a.K[t]);
+    return;
+  }
+  if (w == 0) {  // the producer is not a writer: it never holds the minimum back
+    if (lane == 0) {
+      st_release_cta(&sh.done[0], a.K[t]);
+      tma_produce(a, e, t, j, sh, ring);
+    }
+    return;
+  }
+  switch (e.nin) {
+    case 1: tma_nout<DT, 1, SGD>(a, e, t, w, w - 1, W - 1, sh, ring); break;
+    case 2: tma_nout<DT, 2, SGD>(a, e, t, w, w - 1, W - 1, sh, ring); break;
+    default: tma_nout<DT, 3, SGD>(a, e, t, w, w - 1, W - 1, sh, ring); break;
+  }
+}
+
 template <int DT, bool SGD>
 __device__ void data_warp(const LaunchArgs &a, const TreeParams &p, int role, int t, int j,
                           int w, int W, Shared &sh) {
@@ -730,6 +991,7 @@ __device__ void data_warp(const LaunchArgs &a, const TreeParams &p, int role, in
 template <int DT, bool SYS, bool SGD, int MAXT>
 __global__ void __launch_bounds__(MAXT, kMinBlocksPerSm) tree_allreduce_kernel(const LaunchArgs a) {
   __shared__ Shared sh;
+  extern __shared__ __align__(128) char tma_ring[];  // kTmaRing bytes on the TMA datapath
   const Task task = a.tasks[blockIdx.x];
   const TreeParams &p = a.params[task.local_rank * a.ntrees + task.tree];
   const int warp = threadIdx.x >> 5;
@@ -741,11 +1003,20 @@ __global__ void __launch_bounds__(MAXT, kMinBlocksPerSm) tree_allreduce_kernel(c
   if (threadIdx.x == 0) {
     sh.ready = 0;
     sh.abort = 0;
+    if (a.tma) {
+      for (int s = 0; s < kTmaMaxStages; ++s) {
+        mbar_init(&sh.full[s], 1);
+        mbar_init(&sh.empty[s], W - 1);
+      }
+      asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
   }
   if (threadIdx.x < kMaxDataWarps) sh.done[threadIdx.x] = 0;
   __syncthreads();
   if (warp == 0)
     control_warp<SYS>(a, p, task.role, task.tree, task.channel, W, sh);
+  else if (a.tma)
+    tma_data_warp<DT, SGD>(a, p, task.role, task.tree, task.channel, warp - 1, W, sh, tma_ring);
   else
     data_warp<DT, SGD>(a, p, task.role, task.tree, task.channel, warp - 1, W, sh);
 }
@@ -776,10 +1047,16 @@ __global__ void gate_kernel(const GateArgs g) {
 
 template <int DT, bool SYS, bool SGD>
 int launch_t(const LaunchArgs &a, int grid, int threads, cudaStream_t s) {
-  if (threads <= 256)
-    tree_allreduce_kernel<DT, SYS, SGD, 256><<<grid, threads, 0, s>>>(a);
-  else
-    tree_allreduce_kernel<DT, SYS, SGD, kMaxThreads><<<grid, threads, 0, s>>>(a);
+  const size_t smem = a.tma ? kTmaRing : 0;
+  if (threads <= 256) {
+    auto *fn = tree_allreduce_kernel<DT, SYS, SGD, 256>;
+    if (smem) cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    fn<<<grid, threads, smem, s>>>(a);
+  } else {
+    auto *fn = tree_allreduce_kernel<DT, SYS, SGD, kMaxThreads>;
+    if (smem) cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    fn<<<grid, threads, smem, s>>>(a);
+  }
   return static_cast<int>(cudaGetLastError());
 }
 
@@ -837,7 +1114,8 @@ int launch_gate(const uint64_t *const *counters, const uint64_t *targets, int n,
   return static_cast<int>(cudaGetLastError());
 }
 
-int query_max_blocks_per_sm(int dtype, bool sys_scope, bool sgd, int threads, int *blocks) {
+int query_max_blocks_per_sm(int dtype, bool sys_scope, bool sgd, int threads, int tma,
+                            int *blocks) {
   const void *fn = nullptr;
   if (sgd) {
     fn = sys_scope ? kernel_ptr<kFloat32, true, true>(threads) : kernel_ptr<kFloat32, false, true>(threads);
@@ -855,7 +1133,13 @@ int query_max_blocks_per_sm(int dtype, bool sys_scope, bool sgd, int threads, in
         break;
     }
   }
-  return static_cast<int>(cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks, fn, threads, 0));
+  const size_t smem = tma ? kTmaRing : 0;
+  if (smem) {
+    const int rc = static_cast<int>(
+        cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+    if (rc != cudaSuccess) return rc;
+  }
+  return static_cast<int>(cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks, fn, threads, smem));
 }
 
 }  // namespace ccube

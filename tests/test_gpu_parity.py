@@ -407,3 +407,58 @@ def test_fused_sgd_rejects_non_fp32(comm):
         ccube.allreduce_tree_local(ts)
     assert e.value.code == ccube.ERR_INVALID_ARG
     ccube.gradq_set_sgd(None)
+
+
+@pytest.mark.parametrize("P", [2, 3, 5, 8])
+@pytest.mark.parametrize("kind", ["single", "double", "rotated"])
+@pytest.mark.parametrize("dtype", ["int32", "float32", "bfloat16"])
+@pytest.mark.parametrize("transport", ["pull", "push"])
+def test_parity_tma_datapath(comm, P, kind, dtype, transport):
+    """The TMA datapath (cp.async.bulk shared-memory ring, consumer warps combine from
+    shared memory) is bit-exact to the oracle: several chunks, ragged tail (< 16 B)
+    and slices longer than one ring stage (8 KB) at 2 channels."""
+    chunk = 48 * 1024
+    comm(P, kind, chunk, channels=2, transport=transport)
+    ccube.set_datapath("tma")
+    assert ccube.get_info()["datapath"] == 1
+    E = chunk // arith.ELEM_SIZE[dtype]
+    count = 5 * E + 7 if dtype == "bfloat16" else 5 * E + 3
+    xs, outs = _run(P, kind, dtype, count, chunk)
+    ref = oar.reference(xs, kind, chunk, dtype)[0]
+    for r in range(P):
+        assert np.array_equal(outs[r], ref), f"rank {r}"
+
+
+@pytest.mark.parametrize("datapath", ["lsu", "tma"])
+@pytest.mark.parametrize("prefetch", [1, 4, 64])
+def test_parity_prefetch(comm, datapath, prefetch):
+    """L2 prefetch of the raw inputs is a hint: results stay bit-exact at any distance
+    (including one beyond the last chunk), across two epochs."""
+    chunk = 16 * 1024
+    comm(8, "double", chunk, channels=3)
+    ccube.set_datapath(datapath)
+    ccube.set_prefetch(prefetch)
+    assert ccube.get_info()["prefetch"] == prefetch
+    count = 9 * chunk // 4 + 5
+    for seed in (5, 6):
+        xs, outs = _run(8, "double", "float32", count, chunk, seed=seed)
+        ref = oar.reference(xs, "double", chunk, "float32")[0]
+        for r in range(8):
+            assert np.array_equal(outs[r], ref), f"rank {r} seed {seed}"
+
+
+def test_parity_full_size_tma(comm):
+    """configs[1] in the bench's launch configuration (P = 8, single tree, C1, auto
+    channels) on the TMA datapath: sampled chunks bit-exact vs the oracle, every rank
+    identical."""
+    P, chunk = 8, 256 << 10
+    comm(P, "single", chunk)
+    ccube.set_datapath("tma")
+    count, ends, ts = _full_size(P, "single", "float32", "resnet50", chunk)
+    K = partition.num_chunks(count, chunk, 4)
+    for c in (0, 1, 200, K - 2, K - 1):
+        lo, hi, want = oracle_chunk(P, "single", chunk, "float32", count, c, layer_ends=ends)
+        for r in (0, 2, 7):
+            assert np.array_equal(to_numpy(ts[r][lo:hi], "float32"), want), (c, r)
+    for r in range(1, P):
+        assert torch.equal(ts[r], ts[0])

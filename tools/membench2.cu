@@ -14,6 +14,7 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 #include <stdio.h>
+#include <stdlib.h>
 #include <vector>
 
 #define CK(x)                                                                          \
@@ -297,6 +298,21 @@ int main() {
     b.dst[i] = p[3 + i];
   }
   const int g2 = 2 * sms;
+  if (getenv("MB2_PARTIAL")) {
+    // per-CTA throughput when only part of the machine streams (the tree kernel's heavy
+    // stage: 82 of 291 CTAs carry 6 of the 8 DRAM read streams at P=8)
+    for (int g : {41, 82, 164}) {
+      run_lsu<3, 1, 4, false>(b, g, 288);
+      run_lsu<3, 1, 2, true>(b, g, 288);
+      run_tma_combine<3, 1, 4, 8192>(b, g, 288);
+      run_tma_combine<3, 1, 6, 8192>(b, g, 288);
+      run_tma_combine<3, 1, 4, 16384>(b, g, 288);
+      run_lsu<1, 2, 8, false>(b, g, 288);
+      run_tma_copy<2, 4, 16384>(b, g);
+      run_tma_copy<2, 8, 16384>(b, g);
+    }
+    return 0;
+  }
   // copies 1 -> 1, 1 -> 2
   run_lsu<1, 1, 8, false>(b, g2, 288);
   run_lsu<1, 1, 4, true>(b, g2, 288);
