@@ -47,10 +47,8 @@ def parse():
     p.add_argument("--chunk-bytes", type=int, default=256 << 10)
     p.add_argument("--channels", type=int, default=0)
     p.add_argument("--threads", type=int, default=0)
-    p.add_argument("--datapath", choices=["tma", "lsu"], default=None,
+    p.add_argument("--datapath", choices=["auto", "tma", "lsu"], default=None,
                    help="data-warp datapath (default: the library's, CCUBE_DATAPATH)")
-    p.add_argument("--prefetch", type=int, default=None,
-                   help="L2 prefetch distance in chunks (default: the library's, CCUBE_PREFETCH)")
     p.add_argument("--e2e-steps", type=int, default=5)
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-cpu-baseline", action="store_true")
@@ -249,8 +247,6 @@ def run_ccube(a):
         ccube.set_threads(a.threads)
     if a.datapath:
         ccube.set_datapath(a.datapath)
-    if a.prefetch is not None:
-        ccube.set_prefetch(a.prefetch)
     ccube.set_overlap(bool(a.overlap))
     stream = torch.cuda.Stream()
 
@@ -383,8 +379,7 @@ def run_ccube(a):
             "dtype": _dt(a.dtype), "data": "synthetic",
             "config": dict(_config(a, P, nbytes), channels=info["last_channels"],
                            ctas=info["last_ctas"], threads=info["threads"],
-                           datapath={0: "lsu", 1: "tma"}[info["datapath"]],
-                           prefetch_chunks=info["prefetch"],
+                           datapath="tma" if info["last_tma"] else "lsu",
                            l2="inputs (P x bytes_per_rank) larger than L2 and restored from a "
                               "pristine copy between timed steps (flushes L2)"),
             "algbw": alg, "busbw_frac_of_900": bw / NVLINK_NOMINAL_GBS,

@@ -186,22 +186,17 @@ CCUBE_API ccube_result_t ccube_set_overlap(int on);
 CCUBE_API ccube_result_t ccube_set_channels(int channels);
 CCUBE_API ccube_result_t ccube_set_threads(int threads);
 
-/* Datapath of the data warps (values are bitwise identical for both; all ranks
- * must agree).  TMA: one data warp streams every source block into a
- * 96 KB shared-memory ring with cp.async.bulk and the other data warps combine
- * from it (needs >= 2 data warps; with one the LSU path runs).  LSU (default): each
- * data warp keeps its own 128-bit loads in flight in registers.  CCUBE_DATAPATH env sets the
- * initial value.  Errors: NOT_INITIALIZED, INVALID_ARG. */
+/* Datapath of the data warps (values are bitwise identical for every choice; all
+ * ranks must agree).  LSU: each data warp keeps its own 128-bit loads in flight in
+ * registers.  TMA: one data warp streams every source block into a 96 KB
+ * shared-memory ring with cp.async.bulk and the other data warps combine from it
+ * (needs >= 2 data warps; with one the LSU path runs).  AUTO (default): TMA for the
+ * rotated tree set, LSU otherwise (measured).  CCUBE_DATAPATH env
+ * (0 / 1) sets the initial value.  Errors: NOT_INITIALIZED, INVALID_ARG. */
+#define CCUBE_DATAPATH_AUTO (-1)
 #define CCUBE_DATAPATH_LSU 0
 #define CCUBE_DATAPATH_TMA 1
 CCUBE_API ccube_result_t ccube_set_datapath(int datapath);
-
-/* L2 prefetch distance of the reduce-up tasks, in chunks (0 = off; CCUBE_PREFETCH env,
- * default 0).  The control warp of an UP task keeps this many chunks of its raw
- * inputs (own buffer, pulled leaves' buffers) in flight as bulk L2 prefetches ahead
- * of its data warps.  A hint only: values are bitwise identical for every setting.
- * Errors: NOT_INITIALIZED, INVALID_ARG (chunks < 0 or > 1024). */
-CCUBE_API ccube_result_t ccube_set_prefetch(int chunks);
 
 /* Edge transport (physical-topology awareness, cf. §IV).  PUSH: a
  * child stores its partial sum into the parent's receive plane (posted NVLink
@@ -231,8 +226,8 @@ typedef struct {
   size_t chunk_bytes;
   uint64_t epoch_base[2];       /* trees 0 and 1 (ROTATED has P trees) */
   int last_channels, last_ctas;
-  int datapath;                 /* CCUBE_DATAPATH_* */
-  int prefetch;                 /* L2 prefetch distance of UP tasks, chunks */
+  int datapath;                 /* configured CCUBE_DATAPATH_* */
+  int last_tma;                 /* 1 = the most recent launch ran the TMA datapath */
 } ccube_info_t;
 CCUBE_API ccube_result_t ccube_get_info(ccube_info_t *info);
 

@@ -32,14 +32,14 @@ _NAMES = {0: "SUCCESS", -1: "INVALID_ARG", -2: "NOT_INITIALIZED", -3: "ALREADY_I
 
 TREE = {"single": 0, "double": 1, "rotated": 2}
 TRANSPORT = {"auto": 0, "push": 1, "pull": 2}
-DATAPATH = {"lsu": 0, "tma": 1}
+DATAPATH = {"auto": -1, "lsu": 0, "tma": 1}
 DTYPE = {"int32": 0, "float32": 1, "bfloat16": 2}
 
 EXPORTS = [
     "ccube_init", "ccube_register_buffers", "ccube_deregister_buffers", "ccube_allreduce_tree",
     "ccube_allreduce_tree_local", "ccube_gradq_set_layers", "ccube_gradq_wait",
     "ccube_gradq_wait_local", "ccube_gradq_set_sgd", "ccube_set_overlap", "ccube_set_channels", "ccube_set_threads",
-    "ccube_set_trace", "ccube_set_transport", "ccube_set_datapath", "ccube_set_prefetch", "ccube_finalize", "ccube_last_error", "ccube_get_info",
+    "ccube_set_trace", "ccube_set_transport", "ccube_set_datapath", "ccube_finalize", "ccube_last_error", "ccube_get_info",
     "ccube_tree_parents",
 ]
 
@@ -66,7 +66,7 @@ class Info(ctypes.Structure):
                 ("channels", ctypes.c_int), ("threads", ctypes.c_int), ("overlap", ctypes.c_int),
                 ("transport", ctypes.c_int), ("chunk_bytes", ctypes.c_size_t), ("epoch_base", ctypes.c_uint64 * 2),
                 ("last_channels", ctypes.c_int), ("last_ctas", ctypes.c_int),
-                ("datapath", ctypes.c_int), ("prefetch", ctypes.c_int)]
+                ("datapath", ctypes.c_int), ("last_tma", ctypes.c_int)]
 
 
 _lib = None
@@ -98,7 +98,6 @@ def lib() -> ctypes.CDLL:
             "ccube_set_trace": [vp, sz],
             "ccube_set_transport": [i],
             "ccube_set_datapath": [i],
-            "ccube_set_prefetch": [i],
             "ccube_finalize": [],
             "ccube_get_info": [ctypes.POINTER(Info)],
             "ccube_tree_parents": [i, i, i, ctypes.POINTER(i)],
@@ -294,13 +293,9 @@ def set_transport(mode: str) -> None:
 
 
 def set_datapath(mode: str) -> None:
-    """'lsu' (register-staged, default) or 'tma' (cp.async.bulk shared-memory ring)."""
+    """'auto' (default: TMA for the rotated tree set), 'lsu' (register-staged) or 'tma'
+    (cp.async.bulk shared-memory ring)."""
     _check(lib().ccube_set_datapath(DATAPATH[mode]), "ccube_set_datapath")
-
-
-def set_prefetch(chunks: int) -> None:
-    """L2 prefetch distance (chunks) of the reduce-up tasks' raw inputs; 0 = off."""
-    _check(lib().ccube_set_prefetch(chunks), "ccube_set_prefetch")
 
 
 def set_trace(trace_tensor, kmax: int) -> None:

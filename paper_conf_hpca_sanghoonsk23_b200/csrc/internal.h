@@ -72,8 +72,6 @@ struct TreeParams {
   int child_interior[kMaxChildren]; // child has children: its buffer is re-read (DOWN)
   char *w;                          // own fp32 weights (fused SGD, f2), same layout as buf
   uint64_t *upd;                    // own "weights updated" counter (channel 0)
-  uint32_t pf_mask;                 // bit q: up_src[q] is a raw input (own buf, a pulled
-                                    // leaf's buf), readable from the start: L2 prefetch
 };
 
 // UPDATE: a leaf's fused-SGD task (f2) — waits for its chunks to land, then
@@ -108,8 +106,8 @@ struct LaunchArgs {
   int sgd;                    // 1 = fused SGD update at landing (fp32 only)
   float sgd_alpha;            // w <- w - sgd_alpha * g
   int tma;                    // datapath: 0 = register-staged LSU, 1 = TMA bulk-load ring
-  int prefetch;               // UP tasks prefetch raw inputs this many chunks ahead (0 = off)
   int elem_size;              // bytes per element (2 or 4)
+  int split_control;          // 1 = separate poll and publish warps (warps 0, 1)
 };
 
 // Kernel launcher (tree_allreduce.cu).  Returns a cudaError_t as int.

@@ -166,8 +166,9 @@ struct Comm {
   int last_channels = 0;
   int last_ctas = 0;
   int l2_hints = 1;
-  int datapath = CCUBE_DATAPATH_LSU;  // CCUBE_DATAPATH env / ccube_set_datapath
-  int prefetch = 0;                   // CCUBE_PREFETCH env: chunks of L2 prefetch ahead
+  int datapath = CCUBE_DATAPATH_AUTO;  // CCUBE_DATAPATH env / ccube_set_datapath
+  int last_tma = 0;
+  int split_control = 1;              // CCUBE_SPLIT_CONTROL env: poll and publish warps
   bool sgd = false;                 // fused SGD update (f2)
   float sgd_alpha = 0.0f;
   size_t sgd_bytes = 0;
@@ -303,7 +304,6 @@ ccube_result_t build_params(Registration *R) {
       memset(&p, 0, sizeof p);
       p.buf = R->bufs[i];
       p.up_src[0] = R->bufs[i];
-      p.pf_mask = 1u;  // my own input
       p.nchild = tr.nchild[r];
       p.is_root = tr.parent[r] < 0;
       p.self_local = i;
@@ -343,7 +343,6 @@ ccube_result_t build_params(Registration *R) {
         p.child_interior[s] = tr.nchild[c] > 0;
         if (edge_is_pull(c, r)) {
           p.up_src[1 + s] = R->world_buf[c];
-          if (tr.nchild[c] == 0) p.pf_mask |= 2u << s;  // a pulled leaf: its raw input
         } else {
           if (!R->recv[i]) return fail(CCUBE_ERR_BOOTSTRAP, "receive plane missing");
           p.up_src[1 + s] = R->recv[i] + static_cast<size_t>(s) * R->plane;
@@ -513,9 +512,14 @@ ccube_result_t allreduce_impl(void *const *bufs, size_t count, ccube_dtype_t dty
   if (K > 0xffffffffull) return fail(CCUBE_ERR_INVALID_ARG, "too many chunks");
 
   // all CTAs spin on each other: they must be co-resident
-  const int cta_threads = g.threads + 32;  // data warps + the control warp
+  const int nctl = g.split_control ? 2 : 1;
+  const int cta_threads = g.threads + 32 * nctl;  // data warps + the control warp(s)
   // the TMA datapath needs a producer and at least one consumer data warp
-  const int tma = g.datapath == CCUBE_DATAPATH_TMA && g.threads >= 64 ? 1 : 0;
+  // (AUTO: TMA for the rotated tree set, whose P trees leave few channels and long
+  // slices per chunk; the register-staged LSU path for the single and double tree)
+  const bool want_tma = g.datapath == CCUBE_DATAPATH_TMA ||
+                        (g.datapath == CCUBE_DATAPATH_AUTO && g.ntrees > 2);
+  const int tma = want_tma && g.threads >= 64 ? 1 : 0;
   auto key = std::make_pair((int)dtype * 2 + (g.sgd ? 1 : 0) + 8 * tma, cta_threads);
   if (!g.max_blocks.count(key)) {
     int b = 0;
@@ -560,7 +564,7 @@ ccube_result_t allreduce_impl(void *const *bufs, size_t count, ccube_dtype_t dty
   a.sgd = g.sgd ? 1 : 0;
   a.sgd_alpha = g.sgd_alpha;
   a.tma = tma;
-  a.prefetch = g.prefetch;
+  a.split_control = g.split_control;
   a.elem_size = static_cast<int>(es);
   a.params = R->d_params;
 
@@ -581,6 +585,7 @@ ccube_result_t allreduce_impl(void *const *bufs, size_t count, ccube_dtype_t dty
   g.last_channels = J;
   g.last_sgd = g.sgd;
   g.last_ctas = tt->n;
+  g.last_tma = tma;
   for (int t = 0; t < g.ntrees; ++t) {
     g.last_base[t] = g.base[t];
     g.last_K[t] = a.K[t];
@@ -731,11 +736,10 @@ ccube_result_t ccube_init(const ccube_world_t *world, ccube_tree_kind_t tree_kin
   g.transport = transport;
   g.overlap = 1;
   g.l2_hints = env_int("CCUBE_L2_HINTS", 1);
-  g.datapath = env_int("CCUBE_DATAPATH", CCUBE_DATAPATH_LSU) == CCUBE_DATAPATH_TMA
-                   ? CCUBE_DATAPATH_TMA
-                   : CCUBE_DATAPATH_LSU;
-  g.prefetch = env_int("CCUBE_PREFETCH", 0);
-  if (g.prefetch < 0) g.prefetch = 0;
+  g.split_control = env_int("CCUBE_SPLIT_CONTROL", 1) != 0 ? 1 : 0;
+  g.datapath = env_int("CCUBE_DATAPATH", CCUBE_DATAPATH_AUTO);
+  if (g.datapath != CCUBE_DATAPATH_LSU && g.datapath != CCUBE_DATAPATH_TMA)
+    g.datapath = CCUBE_DATAPATH_AUTO;
   g.sys_scope = g.nproc > 1;
   g.timeout_ns = static_cast<uint64_t>(env_int("CCUBE_WATCHDOG_MS", 10000)) * 1000000ull;
   g.use_memop = env_int("CCUBE_GATE_KERNEL", 0) == 0;
@@ -952,18 +956,10 @@ ccube_result_t ccube_set_threads(int threads) {
 ccube_result_t ccube_set_datapath(int datapath) {
   std::lock_guard<std::mutex> lk(g_mu);
   if (!g.init) return fail(CCUBE_ERR_NOT_INITIALIZED, "ccube_init has not been called");
-  if (datapath != CCUBE_DATAPATH_LSU && datapath != CCUBE_DATAPATH_TMA)
+  if (datapath != CCUBE_DATAPATH_LSU && datapath != CCUBE_DATAPATH_TMA &&
+      datapath != CCUBE_DATAPATH_AUTO)
     return fail(CCUBE_ERR_INVALID_ARG, "datapath %d out of range", datapath);
   g.datapath = datapath;
-  return CCUBE_SUCCESS;
-}
-
-ccube_result_t ccube_set_prefetch(int chunks) {
-  std::lock_guard<std::mutex> lk(g_mu);
-  if (!g.init) return fail(CCUBE_ERR_NOT_INITIALIZED, "ccube_init has not been called");
-  if (chunks < 0 || chunks > 1024)
-    return fail(CCUBE_ERR_INVALID_ARG, "prefetch %d out of range [0, 1024]", chunks);
-  g.prefetch = chunks;
   return CCUBE_SUCCESS;
 }
 
@@ -1033,7 +1029,7 @@ ccube_result_t ccube_get_info(ccube_info_t *info) {
   info->last_channels = g.last_channels;
   info->last_ctas = g.last_ctas;
   info->datapath = g.datapath;
-  info->prefetch = g.prefetch;
+  info->last_tma = g.last_tma;
   return CCUBE_SUCCESS;
 }
 

@@ -36,7 +36,7 @@
 namespace ccube {
 namespace {
 
-constexpr int kMaxThreads = 288;  // up to 8 data warps + the control warp
+constexpr int kMaxThreads = 320;  // up to 8 data warps + one or two control warps
 constexpr int kMaxDataWarps = 8;
 constexpr int kMinBlocksPerSm = 2;  // two CTAs per SM: <= 112 registers per thread
 
@@ -552,35 +552,6 @@ __device__ __forceinline__ void combine_scalar(const char *const *src, int nin, 
 // each data warp streams its blocks (BlockIter) and reports, through a per-warp
 // "done" counter, the chunk of its next block; the control warp publishes the
 // minimum over the warps downstream.
-// L2 prefetch of an UP task's raw inputs (own buffer, pulled leaves' buffers): they
-// sit in DRAM from the start, so the control warp keeps `a.prefetch` chunks of this
-// channel's slices in flight ahead of the data warps with bulk L2 prefetches (no
-// registers, no shared memory).  The data warps' loads then hit L2: the DRAM latency
-// leaves the critical path of the DRAM-heavy tasks.  Prefetching is only a hint —
-// L2 is the point of coherence, so a line prefetched early is still updated by any
-// later write.
-struct Prefetcher {
-  Geo g;
-  uint32_t k, c;   // next chunk to prefetch, k mod J
-  uint64_t c0;     // its byte offset
-  const char *src; // this lane's source (nullptr = none)
-};
-
-__device__ __forceinline__ void prefetch_l2(const void *ptr, uint32_t bytes) {
-  asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(ptr), "r"(bytes) : "memory");
-}
-
-__device__ __forceinline__ void prefetch_until(Prefetcher &pf, uint32_t upto) {
-  while (pf.k < pf.g.K && pf.k < upto) {
-    const Slice sl = slice_at(pf.g, pf.c, pf.c0);
-    const uint32_t len = sl.len & ~15u;
-    if (pf.src && len) prefetch_l2(pf.src + sl.off, len);
-    ++pf.k;
-    pf.c = pf.c + 1 == pf.g.J ? 0 : pf.c + 1;
-    pf.c0 += pf.g.stride;
-  }
-}
-
 template <bool SYS>
 __device__ void control_warp(const LaunchArgs &a, const TreeParams &p, int role, int t, int j,
                              int W, Shared &sh) {
@@ -588,17 +559,6 @@ __device__ void control_warp(const LaunchArgs &a, const TreeParams &p, int role,
   const uint32_t K = a.K[t];
   const uint64_t base = a.base[t];
   const int stride = j * kFlagStrideU64;
-  const bool do_pf = role == kRoleUp && a.prefetch > 0 && lane <= p.nchild &&
-                     ((p.pf_mask >> lane) & 1u);
-  Prefetcher pf;
-  if (do_pf) {
-    pf.g = a.elem_size == 2 ? make_geo<2>(a, t, j) : make_geo<4>(a, t, j);
-    pf.k = 0;
-    pf.c = 0;
-    pf.c0 = pf.g.first;
-    pf.src = p.up_src[lane];
-    prefetch_until(pf, static_cast<uint32_t>(a.prefetch));
-  }
   const uint64_t *up = nullptr;
   if (role == kRoleUp) {
     if (lane < p.nchild) up = p.head_in[lane] + stride;
@@ -633,7 +593,6 @@ __device__ void control_warp(const LaunchArgs &a, const TreeParams &p, int role,
       if (lane == 0) publish<SYS>(a, p, role, t, j, pub, static_cast<uint32_t>(d), base);
       pub = static_cast<uint32_t>(d);
       moved = true;
-      if (do_pf) prefetch_until(pf, pub + static_cast<uint32_t>(a.prefetch));
     }
     if (moved) {
       watch_reset(wd);
@@ -644,6 +603,87 @@ __device__ void control_warp(const LaunchArgs &a, const TreeParams &p, int role,
         st_relaxed<SYS>(p.upd + stride, ~0ull);
       }
       return;
+    }
+  }
+  leaf_wait<SYS>(a, p, role, t, j);
+}
+
+// Split control (a.split_control): the two duties of control_warp run on two warps,
+// so neither waits for the other.  The poll warp's loop is one global acquire round
+// trip; the publish warp's loop is a shared-memory read, so a finished chunk is
+// released downstream after the fence alone instead of after up to one upstream
+// poll as well (the per-hop latency, alpha, that sets the pipeline's fill and drain).
+template <bool SYS>
+__device__ void poll_warp(const LaunchArgs &a, const TreeParams &p, int role, int t, int j,
+                          Shared &sh) {
+  const int lane = threadIdx.x & 31;
+  const uint32_t K = a.K[t];
+  const uint64_t base = a.base[t];
+  const int stride = j * kFlagStrideU64;
+  const uint64_t *up = nullptr;
+  if (role == kRoleUp) {
+    if (lane < p.nchild) up = p.head_in[lane] + stride;
+  } else if (lane == 0) {
+    up = p.enq + stride;
+  }
+  const bool hold_all = role == kRoleDown && p.is_root;  // B-mode root (Obs #1)
+  uint64_t ready = (role == kRoleUp && p.nchild == 0) ? K : 0;  // a leaf's input is ready
+  if (lane == 0) st_release_cta(&sh.ready, ready);
+  Watch wd;
+  watch_reset(wd);
+  while (ready < K) {
+    uint64_t v = up ? ld_acquire<SYS>(up) : ~0ull;
+    v = warp_min(v);
+    uint64_t r = v > base ? v - base : 0;
+    if (r > K) r = K;
+    if (hold_all && r < K) r = 0;
+    if (r > ready) {
+      __syncwarp();  // every lane's acquire happens before lane 0's release below
+      ready = r;
+      if (lane == 0) st_release_cta(&sh.ready, ready);
+      watch_reset(wd);
+    } else {
+      if (*reinterpret_cast<volatile int *>(&sh.abort)) return;
+      if (!watch_tick(wd, a, base + ready + 1, 0)) {
+        if (lane == 0) {
+          *reinterpret_cast<volatile int *>(&sh.abort) = 1;
+          st_relaxed<SYS>(p.enq + stride, ~0ull);  // release gradient-queue waiters
+          st_relaxed<SYS>(p.upd + stride, ~0ull);
+        }
+        return;
+      }
+    }
+  }
+}
+
+template <bool SYS>
+__device__ void publish_warp(const LaunchArgs &a, const TreeParams &p, int role, int t, int j,
+                             int W, Shared &sh) {
+  const int lane = threadIdx.x & 31;
+  const uint32_t K = a.K[t];
+  const uint64_t base = a.base[t];
+  const int stride = j * kFlagStrideU64;
+  uint32_t pub = 0;
+  Watch wd;
+  watch_reset(wd);
+  while (pub < K) {
+    uint64_t d = lane < W ? ld_acquire_cta(&sh.done[lane]) : ~0ull;
+    d = warp_min(d);
+    if (d > pub) {
+      __syncwarp();
+      if (lane == 0) publish<SYS>(a, p, role, t, j, pub, static_cast<uint32_t>(d), base);
+      pub = static_cast<uint32_t>(d);
+      watch_reset(wd);
+    } else {
+      if (*reinterpret_cast<volatile int *>(&sh.abort)) return;
+      if (!watch_tick(wd, a, base + pub + 1, base + pub)) {
+        if (lane == 0) {
+          *reinterpret_cast<volatile int *>(&sh.abort) = 1;
+          st_relaxed<SYS>(p.enq + stride, ~0ull);
+          st_relaxed<SYS>(p.upd + stride, ~0ull);
+        }
+        return;
+      }
     }
   }
   leaf_wait<SYS>(a, p, role, t, j);
@@ -999,7 +1039,8 @@ __global__ void __launch_bounds__(MAXT, kMinBlocksPerSm) tree_allreduce_kernel(c
     if (warp == 0) pulled_leaf<SYS>(a, p, task.tree);
     return;
   }
-  const int W = (blockDim.x >> 5) - 1;
+  const int nctl = a.split_control ? 2 : 1;  // control warps ahead of the data warps
+  const int W = (blockDim.x >> 5) - nctl;
   if (threadIdx.x == 0) {
     sh.ready = 0;
     sh.abort = 0;
@@ -1013,12 +1054,18 @@ __global__ void __launch_bounds__(MAXT, kMinBlocksPerSm) tree_allreduce_kernel(c
   }
   if (threadIdx.x < kMaxDataWarps) sh.done[threadIdx.x] = 0;
   __syncthreads();
-  if (warp == 0)
-    control_warp<SYS>(a, p, task.role, task.tree, task.channel, W, sh);
-  else if (a.tma)
-    tma_data_warp<DT, SGD>(a, p, task.role, task.tree, task.channel, warp - 1, W, sh, tma_ring);
-  else
-    data_warp<DT, SGD>(a, p, task.role, task.tree, task.channel, warp - 1, W, sh);
+  if (warp == 0) {
+    if (a.split_control)
+      poll_warp<SYS>(a, p, task.role, task.tree, task.channel, sh);
+    else
+      control_warp<SYS>(a, p, task.role, task.tree, task.channel, W, sh);
+  } else if (warp < nctl) {
+    publish_warp<SYS>(a, p, task.role, task.tree, task.channel, W, sh);
+  } else if (a.tma) {
+    tma_data_warp<DT, SGD>(a, p, task.role, task.tree, task.channel, warp - nctl, W, sh, tma_ring);
+  } else {
+    data_warp<DT, SGD>(a, p, task.role, task.tree, task.channel, warp - nctl, W, sh);
+  }
 }
 
 struct GateArgs {
@@ -1071,7 +1118,9 @@ const void *kernel_ptr(int threads) {
 
 int launch_tree_allreduce(const LaunchArgs &args, int dtype, bool sys_scope, int grid,
                           int threads, void *stream) {
-  if (threads > kMaxThreads || threads < 64 || threads % 32 || threads / 32 - 1 > kMaxDataWarps)
+  const int nctl = args.split_control ? 2 : 1;
+  if (threads > kMaxThreads || threads < 32 * (nctl + 1) || threads % 32 ||
+      threads / 32 - nctl > kMaxDataWarps)
     return cudaErrorInvalidValue;
   cudaStream_t s = static_cast<cudaStream_t>(stream);
   if (args.sgd) {

@@ -44,6 +44,7 @@ def test_tree_parents_rejects_bad_args():
 
 def test_calls_before_init_fail_cleanly():
     for fn, args in [(ccube.set_overlap, (1,)), (ccube.set_channels, (4,)),
+                     (ccube.set_datapath, ("tma",)), (ccube.set_datapath, ("auto",)),
                      (ccube.gradq_set_layers, ([1, 2],)), (ccube.finalize, ())]:
         with pytest.raises(ccube.CCubeError) as e:
             fn(*args)
