@@ -36,6 +36,13 @@
 namespace ccube {
 namespace {
 
+#ifndef CCUBE_U_COMBINE
+#define CCUBE_U_COMBINE 4  // 16-byte vectors per lane per source in flight (combines)
+#endif
+#ifndef CCUBE_U_COPY
+#define CCUBE_U_COPY 8     // ... (copies)
+#endif
+
 constexpr int kMaxThreads = 320;  // up to 8 data warps + one or two control warps
 constexpr int kMaxDataWarps = 8;
 constexpr int kMinBlocksPerSm = 2;  // two CTAs per SM: <= 112 registers per thread
@@ -787,7 +794,8 @@ __device__ void lsu_stream(const LaunchArgs &a, const Endpoints &e, int t, int j
 template <int DT, int NIN, bool SGD>
 __device__ __forceinline__ void lsu_nout(const LaunchArgs &a, const Endpoints &e, int t, int j,
                                          int w, int W, Shared &sh) {
-  constexpr int U = NIN == 1 ? 8 : 4;  // block = 4 KB (copies) or 2 KB (combines)
+  // block = 4 KB (copies) or 2 KB (combines); build-time overrides for experiments
+  constexpr int U = NIN == 1 ? CCUBE_U_COPY : CCUBE_U_COMBINE;
   if constexpr (SGD && DT == kFloat32 && NIN <= 2) {
     if (e.sgd) {  // root UP (NIN 2), interior DOWN and leaf UPDATE (NIN 1); U = 4 (2 KB)
       switch (e.nout) {
