@@ -40,7 +40,7 @@ namespace {
 #define CCUBE_U_COMBINE 4  // 16-byte vectors per lane per source in flight (combines)
 #endif
 #ifndef CCUBE_U_COPY
-#define CCUBE_U_COPY 8     // ... (copies)
+#define CCUBE_U_COPY 4     // ... (copies; 8 measured 1% slower, v16)
 #endif
 
 constexpr int kMaxThreads = 320;  // up to 8 data warps + one or two control warps
@@ -794,7 +794,7 @@ __device__ void lsu_stream(const LaunchArgs &a, const Endpoints &e, int t, int j
 template <int DT, int NIN, bool SGD>
 __device__ __forceinline__ void lsu_nout(const LaunchArgs &a, const Endpoints &e, int t, int j,
                                          int w, int W, Shared &sh) {
-  // block = 4 KB (copies) or 2 KB (combines); build-time overrides for experiments
+  // block = 2 KB (copies and combines); build-time overrides for experiments
   constexpr int U = NIN == 1 ? CCUBE_U_COPY : CCUBE_U_COMBINE;
   if constexpr (SGD && DT == kFloat32 && NIN <= 2) {
     if (e.sgd) {  // root UP (NIN 2), interior DOWN and leaf UPDATE (NIN 1); U = 4 (2 KB)
