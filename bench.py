@@ -53,6 +53,9 @@ def parse():
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--no-clocks", action="store_true")
+    p.add_argument("--no-nccl", action="store_true",
+                   help="N>1: skip the NCCL Ring/Tree/default comparison on the same buffer")
+    p.add_argument("--nccl-steps", type=int, default=20)
     p.add_argument("--cpu-sample-chunks", type=int, default=0,
                    help="chunks per step for the oracle (0 = auto)")
     p.add_argument("--mode", choices=["allreduce", "iter"], default="allreduce",
@@ -360,6 +363,11 @@ def run_ccube(a):
                "sample": f"oracle.allreduce.replay on the first {nch} chunks ({sb} B per rank) "
                          f"of the {a.workload} gradient set, P={P}, {a.tree} tree; {dt:.2f} s"}
 
+    # ---- NCCL on the same box and buffer (the comparison baseline, N>1 only)
+    nccl = None
+    if multi and not a.no_nccl:
+        nccl = nccl_compare(a, dev, bufs[0], pristine[0], nbytes, P, stream)
+
     info = ccube.get_info()
     ccube.finalize()
     iteration = None
@@ -388,6 +396,8 @@ def run_ccube(a):
             "ms_per_step_p10_p50_p90": [float(np.percentile(ms, q)) for q in (10, 50, 90)],
             "iteration": iteration,
         }
+        if nccl is not None:
+            line["nccl"] = nccl
         print(json.dumps(line), flush=True)
     if multi:
         dist.destroy_process_group()
@@ -519,6 +529,55 @@ def run_iteration(a, P, log=None):
     out["exposed_cut_CC_vs_B"] = cut("CC", "B")
     out["exposed_cut_C2_vs_B"] = cut("C2", "B")      # chaining alone
     out["exposed_cut_CC_vs_C1"] = cut("CC", "C1")    # chaining on top of the overlapped tree
+    return out
+
+
+def nccl_compare(a, dev, buf, pristine, nbytes, P, stream):
+    """NCCL AllReduce (sum) on the same buffer, dtype and timing protocol as the
+    C-Cube arm: Ring, Tree and NCCL's own default choice.  NCCL_ALGO is read when a
+    communicator is created, so each algorithm gets a fresh group created after the
+    variable is set.  Returns {algo: {"busbw": GB/s, "ms_per_step": ms}}."""
+    import torch
+    import torch.distributed as dist
+
+    out = {}
+    saved = os.environ.get("NCCL_ALGO")
+    for algo in ("Ring", "Tree", "default"):
+        if algo == "default":
+            os.environ.pop("NCCL_ALGO", None)
+        else:
+            os.environ["NCCL_ALGO"] = algo
+        try:
+            g = dist.new_group(backend="nccl")
+            with torch.cuda.stream(stream):
+                for _ in range(max(3, a.warmup)):
+                    buf.copy_(pristine)
+                    dist.all_reduce(buf, group=g)
+            torch.cuda.synchronize()
+            evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+                   for _ in range(a.nccl_steps)]
+            dist.barrier()
+            torch.cuda.synchronize()
+            with torch.cuda.stream(stream):
+                for s, e in evs:
+                    buf.copy_(pristine)
+                    s.record(stream)
+                    dist.all_reduce(buf, group=g)
+                    e.record(stream)
+            torch.cuda.synchronize()
+            t = torch.tensor([sum(s.elapsed_time(e) for s, e in evs)], device=dev)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            ms = t.item() / a.nccl_steps
+            bw, alg = busbw(nbytes, ms / 1e3, P)
+            out[algo] = {"busbw": bw, "algbw": alg, "ms_per_step": ms,
+                         "busbw_frac_of_900": bw / NVLINK_NOMINAL_GBS}
+            dist.destroy_process_group(g)
+        except Exception as e:  # noqa: BLE001 — reported in the line, the C-Cube arm stands
+            out[algo] = {"error": repr(e)}
+    if saved is None:
+        os.environ.pop("NCCL_ALGO", None)
+    else:
+        os.environ["NCCL_ALGO"] = saved
     return out
 
 

@@ -169,6 +169,7 @@ struct Comm {
   int datapath = CCUBE_DATAPATH_AUTO;  // CCUBE_DATAPATH env / ccube_set_datapath
   int last_tma = 0;
   int split_control = 1;              // CCUBE_SPLIT_CONTROL env: poll and publish warps
+  int task_order = 0;                 // CCUBE_TASK_ORDER env: block -> task placement
   bool sgd = false;                 // fused SGD update (f2)
   float sgd_alpha = 0.0f;
   size_t sgd_bytes = 0;
@@ -416,6 +417,40 @@ Registration *find_registration(void *const *bufs, size_t bytes) {
   return nullptr;
 }
 
+// Block -> task placement.  Values never depend on it (every CTA is co-resident and
+// a task's work is fixed by its (rank, tree, role, channel)); only which tasks share
+// an SM does.  The block scheduler fills one CTA per SM before the second, so block
+// b and block b + #SMs usually share an SM.
+//   0: rank-major (the construction order above);
+//   1: channel-major: the tasks of channel j are adjacent, so an SM pair mixes roles;
+//   2: heavy first: tasks that combine children's partials (UP with children, the
+//      DRAM-read-heavy stages) fill the first blocks, copies and leaves the rest, so
+//      an SM rarely hosts two combining tasks.
+int task_weight(const Task &x) {
+  if (x.channel == kAllChannels) return 3;             // pulled leaf: no data
+  if (x.role == kRoleDown || x.role == kRoleUpdate) return 2;  // copy (+ update)
+  const Tree &tr = g.trees[x.tree];
+  const int r = g.rank0 + x.local_rank;
+  if (tr.parent[r] < 0) return 1;                      // root: 2 sources
+  return tr.nchild[r] > 0 ? 0 : 2;                     // interior combine / pushed leaf
+}
+
+void order_tasks(std::vector<Task> &ts) {
+  if (g.task_order == 1) {
+    std::stable_sort(ts.begin(), ts.end(), [](const Task &x, const Task &y) {
+      const int cx = x.channel == kAllChannels ? -1 : x.channel;
+      const int cy = y.channel == kAllChannels ? -1 : y.channel;
+      return cx < cy;
+    });
+  } else if (g.task_order == 2) {
+    std::stable_sort(ts.begin(), ts.end(), [](const Task &x, const Task &y) {
+      const int wx = task_weight(x), wy = task_weight(y);
+      if (wx != wy) return wx < wy;
+      return x.channel < y.channel;
+    });
+  }
+}
+
 ccube_result_t get_tasks(int channels, int overlap, TaskTable **out) {
   auto key = std::make_pair(channels, overlap * 2 + (g.sgd ? 1 : 0));
   auto it = g.tasks.find(key);
@@ -444,6 +479,7 @@ ccube_result_t get_tasks(int channels, int overlap, TaskTable **out) {
           ts.push_back(Task{(int16_t)i, (int16_t)t, (int16_t)kRoleDown, (int16_t)j});
     }
   }
+  order_tasks(ts);
   TaskTable tt;
   tt.n = static_cast<int>(ts.size());
   CUDA_TRY(cudaMalloc(&tt.d_tasks, sizeof(Task) * ts.size()));
@@ -737,6 +773,7 @@ ccube_result_t ccube_init(const ccube_world_t *world, ccube_tree_kind_t tree_kin
   g.overlap = 1;
   g.l2_hints = env_int("CCUBE_L2_HINTS", 1);
   g.split_control = env_int("CCUBE_SPLIT_CONTROL", 1) != 0 ? 1 : 0;
+  g.task_order = env_int("CCUBE_TASK_ORDER", 0);
   g.datapath = env_int("CCUBE_DATAPATH", CCUBE_DATAPATH_AUTO);
   if (g.datapath != CCUBE_DATAPATH_LSU && g.datapath != CCUBE_DATAPATH_TMA)
     g.datapath = CCUBE_DATAPATH_AUTO;
