@@ -56,6 +56,8 @@ def parse():
     p.add_argument("--no-nccl", action="store_true",
                    help="N>1: skip the NCCL Ring/Tree/default comparison on the same buffer")
     p.add_argument("--nccl-steps", type=int, default=20)
+    p.add_argument("--cpu-seconds", type=float, default=10.0,
+                   help="cpu_baseline: repeat the oracle sample until this much CPU work")
     p.add_argument("--cpu-sample-chunks", type=int, default=0,
                    help="chunks per step for the oracle (0 = auto)")
     p.add_argument("--mode", choices=["allreduce", "iter"], default="allreduce",
@@ -139,9 +141,12 @@ class ClockSampler:
 
 
 # ---------------------------------------------------------------- oracle timing
-def oracle_time(P, tree, dtype, workload, chunk_bytes, nchunks, overlap):
+def oracle_time(P, tree, dtype, workload, chunk_bytes, nchunks, overlap, min_seconds=0.0,
+                max_reps=64):
     """Time the CPU oracle's message-passing replay on the first ``nchunks`` chunks
-    of the workload (every rank's data for those chunks)."""
+    of the workload (every rank's data for those chunks), repeated until at least
+    ``min_seconds`` of CPU work (at most ``max_reps`` replays).  Returns (seconds
+    per replay, bytes per rank per replay, replays)."""
     from oracle import allreduce as oar
     from oracle import arith
     from paper_conf_hpca_sanghoonsk23_b200 import inputs, workloads
@@ -149,10 +154,13 @@ def oracle_time(P, tree, dtype, workload, chunk_bytes, nchunks, overlap):
     E = chunk_bytes // arith.ELEM_SIZE[dtype]
     count = min(ends[-1], nchunks * E)
     xs = [inputs.gradients(r, ends[-1], dtype, layer_ends=ends, lo=0, hi=count) for r in range(P)]
-    t0 = time.perf_counter()
-    oar.replay(xs, tree, chunk_bytes, dtype, overlap=bool(overlap))
-    dt = time.perf_counter() - t0
-    return dt, count * arith.ELEM_SIZE[dtype]
+    reps, total = 0, 0.0
+    while reps == 0 or (total < min_seconds and reps < max_reps):
+        t0 = time.perf_counter()
+        oar.replay(xs, tree, chunk_bytes, dtype, overlap=bool(overlap))
+        total += time.perf_counter() - t0
+        reps += 1
+    return total / reps, count * arith.ELEM_SIZE[dtype], reps
 
 
 def busbw(bytes_per_rank, seconds, P):
@@ -171,7 +179,8 @@ def run_reference(a):
         oracle_time(P, a.tree, a.dtype, a.workload, a.chunk_bytes, nchunks, a.overlap)
     total, nbytes = 0.0, 0
     for _ in range(a.steps):
-        dt, nbytes = oracle_time(P, a.tree, a.dtype, a.workload, a.chunk_bytes, nchunks, a.overlap)
+        dt, nbytes, _ = oracle_time(P, a.tree, a.dtype, a.workload, a.chunk_bytes, nchunks,
+                                    a.overlap)
         total += dt
     bw, alg = busbw(nbytes, total / a.steps, P)
     sample = (f"oracle.allreduce.replay on the first {nchunks} chunks ({nbytes} B per rank) of the "
@@ -356,12 +365,15 @@ def run_ccube(a):
 
     cpu = None
     if rank == 0 and not a.no_cpu_baseline:
-        nch = a.cpu_sample_chunks or 64
-        dt, sb = oracle_time(P, a.tree, a.dtype, a.workload, a.chunk_bytes, nch, a.overlap)
+        nch = a.cpu_sample_chunks or 128
+        dt, sb, reps = oracle_time(P, a.tree, a.dtype, a.workload, a.chunk_bytes, nch, a.overlap,
+                                   min_seconds=a.cpu_seconds)
         cbw, _ = busbw(sb, dt, P)
         cpu = {"value": cbw, "unit": "GB/s", "cores": 1, "kind": "oracle",
                "sample": f"oracle.allreduce.replay on the first {nch} chunks ({sb} B per rank) "
-                         f"of the {a.workload} gradient set, P={P}, {a.tree} tree; {dt:.2f} s"}
+                         f"of the {a.workload} gradient set, P={P}, {a.tree} tree, "
+                         f"{'C1' if a.overlap else 'B'}; {reps} replays, {dt * reps:.1f} s of "
+                         f"CPU work ({dt:.3f} s per replay)"}
 
     # ---- NCCL on the same box and buffer (the comparison baseline, N>1 only)
     nccl = None
