@@ -49,7 +49,7 @@ def parse():
     p.add_argument("--threads", type=int, default=0)
     p.add_argument("--datapath", choices=["auto", "tma", "lsu"], default=None,
                    help="data-warp datapath (default: the library's, CCUBE_DATAPATH)")
-    p.add_argument("--e2e-steps", type=int, default=5)
+    p.add_argument("--e2e-steps", type=int, default=10)
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--no-clocks", action="store_true")
@@ -309,31 +309,48 @@ def run_ccube(a):
     if not multi:
         ok = all(torch.equal(bufs[r], bufs[0]) for r in range(1, P))
 
-    # ---- e2e: host buffers -> device -> allreduce -> host, through the public API
+    # ---- e2e: host buffers -> device -> allreduce -> host, through the public API.
+    # Every step copies its inputs in from pinned host memory and its results out.
+    # Two device buffer sets alternate so that step i's device->host copy (second
+    # stream, the other copy engine) overlaps step i+1's host->device copy.
     e2e = None
     if not a.no_e2e:
         outs = [torch.empty_like(h).pin_memory() for h in host]
-        for _ in range(2):
+        sets = [bufs, [torch.empty_like(b) for b in bufs]]
+        dstream = torch.cuda.Stream()
+        ev = lambda: torch.cuda.Event()  # noqa: E731
+        d2h_done = [None, None]
+
+        def e2e_step(i):
+            s_ = i % 2
+            if d2h_done[s_] is not None:          # step i-2's results are out of this set
+                stream.wait_event(d2h_done[s_])
             with torch.cuda.stream(stream):
-                for b, h in zip(bufs, host):
+                for b, h in zip(sets[s_], host):
                     b.copy_(h, non_blocking=True)
-            step()
-            with torch.cuda.stream(stream):
-                for o, b in zip(outs, bufs):
+            if multi:
+                ccube.allreduce_tree(sets[s_][0], stream=stream)
+            else:
+                ccube.allreduce_tree_local(sets[s_], stream=stream)
+            k = ev()
+            k.record(stream)
+            dstream.wait_event(k)
+            with torch.cuda.stream(dstream):
+                for o, b in zip(outs, sets[s_]):
                     o.copy_(b, non_blocking=True)
+            d2h_done[s_] = ev()
+            d2h_done[s_].record(dstream)
+
+        for i in range(2):
+            e2e_step(i)
         torch.cuda.synchronize()
         if multi:
             dist.barrier()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(stream)
-        for _ in range(a.e2e_steps):
-            with torch.cuda.stream(stream):
-                for b, h in zip(bufs, host):
-                    b.copy_(h, non_blocking=True)
-            step()
-            with torch.cuda.stream(stream):
-                for o, b in zip(outs, bufs):
-                    o.copy_(b, non_blocking=True)
+        for i in range(a.e2e_steps):
+            e2e_step(i)
+        stream.wait_stream(dstream)
         e1.record(stream)
         torch.cuda.synchronize()
         e2e_ms = e0.elapsed_time(e1) / a.e2e_steps
@@ -342,9 +359,13 @@ def run_ccube(a):
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
             e2e_ms = t.item()
         ebw, _ = busbw(nbytes, e2e_ms / 1e3, P)
+        ok_e2e = all(torch.equal(o, outs[0]) for o in outs[1:]) if not multi else None
         e2e = {"value": ebw, "unit": "GB/s", "ms_per_step": e2e_ms,
                "h2d_bytes_per_step": nbytes * len(my_ranks),
-               "d2h_bytes_per_step": nbytes * len(my_ranks), "steps": a.e2e_steps}
+               "d2h_bytes_per_step": nbytes * len(my_ranks), "steps": a.e2e_steps,
+               "pipelining": "two device buffer sets; step i's D2H overlaps step i+1's H2D",
+               "ranks_identical": ok_e2e}
+        del sets
 
     # ---- roofline of the (single) kernel
     hbm_peak, peak_src = measured_peaks()
