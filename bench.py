@@ -373,7 +373,7 @@ def run_ccube(a):
         alg_bytes = 2 * P * nbytes   # each rank's buffer read once + written once
         achieved = alg_bytes / (ms_step / 1e3) / 1e9
         roof = {"bound": "hbm", "achieved": achieved, "peak": hbm_peak, "unit": "GB/s",
-                "frac": achieved / hbm_peak, "traffic": _ncu_traffic(),
+                "frac": achieved / hbm_peak, "traffic": _ncu_traffic(a),
                 "peak_source": peak_src,
                 "algorithmic_bytes_per_launch": alg_bytes}
     else:
@@ -627,14 +627,19 @@ def _port_loads(P, kind):
     return loads
 
 
-def _ncu_traffic():
-    """dram bytes per launch from the committed ncu --set full capture, if present."""
+def _ncu_traffic(a):
+    """dram bytes per launch from the committed ncu --set full capture, if it was
+    taken on this line's configuration (the default bench workload), else None."""
     path = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     try:
         with open(path) as f:
-            return json.load(f).get("dram_bytes_per_launch")
+            d = json.load(f)
     except Exception:  # noqa: BLE001
         return None
+    cfg = d.get("config", {})
+    mine = {"workload": a.workload, "tree": a.tree, "ranks": a.ranks, "dtype": a.dtype,
+            "chunk_bytes": a.chunk_bytes, "overlap": a.overlap}
+    return d.get("dram_bytes_per_launch") if cfg == mine else None
 
 
 def _log(msg):
