@@ -141,26 +141,37 @@ class ClockSampler:
 
 
 # ---------------------------------------------------------------- oracle timing
-def oracle_time(P, tree, dtype, workload, chunk_bytes, nchunks, overlap, min_seconds=0.0,
-                max_reps=64):
-    """Time the CPU oracle's message-passing replay on the first ``nchunks`` chunks
-    of the workload (every rank's data for those chunks), repeated until at least
-    ``min_seconds`` of CPU work (at most ``max_reps`` replays).  Returns (seconds
-    per replay, bytes per rank per replay, replays)."""
-    from oracle import allreduce as oar
+def oracle_inputs(P, dtype, workload, chunk_bytes, nchunks):
+    """Every rank's seeded gradients for the first ``nchunks`` chunks of the workload."""
     from oracle import arith
     from paper_conf_hpca_sanghoonsk23_b200 import inputs, workloads
     ends = workloads.layer_ends(workload)
     E = chunk_bytes // arith.ELEM_SIZE[dtype]
     count = min(ends[-1], nchunks * E)
     xs = [inputs.gradients(r, ends[-1], dtype, layer_ends=ends, lo=0, hi=count) for r in range(P)]
+    return xs, count * arith.ELEM_SIZE[dtype]
+
+
+def oracle_replay_time(xs, tree, dtype, chunk_bytes, overlap):
+    """Seconds for one run of the CPU oracle's message-passing replay on ``xs``."""
+    from oracle import allreduce as oar
+    t0 = time.perf_counter()
+    oar.replay(xs, tree, chunk_bytes, dtype, overlap=bool(overlap))
+    return time.perf_counter() - t0
+
+
+def oracle_time(P, tree, dtype, workload, chunk_bytes, nchunks, overlap, min_seconds=0.0,
+                max_reps=64):
+    """Time the CPU oracle's replay on the first ``nchunks`` chunks of the workload
+    (every rank's data for those chunks), repeated until at least ``min_seconds`` of
+    CPU work (at most ``max_reps`` replays).  Returns (seconds per replay, bytes per
+    rank per replay, replays)."""
+    xs, nbytes = oracle_inputs(P, dtype, workload, chunk_bytes, nchunks)
     reps, total = 0, 0.0
     while reps == 0 or (total < min_seconds and reps < max_reps):
-        t0 = time.perf_counter()
-        oar.replay(xs, tree, chunk_bytes, dtype, overlap=bool(overlap))
-        total += time.perf_counter() - t0
+        total += oracle_replay_time(xs, tree, dtype, chunk_bytes, overlap)
         reps += 1
-    return total / reps, count * arith.ELEM_SIZE[dtype], reps
+    return total / reps, nbytes, reps
 
 
 def busbw(bytes_per_rank, seconds, P):
@@ -174,14 +185,13 @@ def run_reference(a):
     if rank != 0:
         return
     P = a.ranks if a.gpus == 1 else a.gpus
-    nchunks = a.cpu_sample_chunks or 16   # 16 chunks x 256 KiB = 4 MiB per rank (configs[0] size)
+    nchunks = a.cpu_sample_chunks or 128  # 128 chunks x 256 KiB = 32 MiB per rank (of 102 MB)
+    xs, nbytes = oracle_inputs(P, a.dtype, a.workload, a.chunk_bytes, nchunks)
     for _ in range(a.warmup):
-        oracle_time(P, a.tree, a.dtype, a.workload, a.chunk_bytes, nchunks, a.overlap)
-    total, nbytes = 0.0, 0
+        oracle_replay_time(xs, a.tree, a.dtype, a.chunk_bytes, a.overlap)
+    total = 0.0
     for _ in range(a.steps):
-        dt, nbytes, _ = oracle_time(P, a.tree, a.dtype, a.workload, a.chunk_bytes, nchunks,
-                                    a.overlap)
-        total += dt
+        total += oracle_replay_time(xs, a.tree, a.dtype, a.chunk_bytes, a.overlap)
     bw, alg = busbw(nbytes, total / a.steps, P)
     sample = (f"oracle.allreduce.replay on the first {nchunks} chunks ({nbytes} B per rank) of the "
               f"{a.workload} gradient set, P={P}, {a.tree} tree, one step = one replay")
