@@ -68,8 +68,8 @@ def parse():
     p.add_argument("--iter-model", choices=["resnet50", "vgg16"], default="resnet50")
     p.add_argument("--iter-fused-sgd", action="store_true",
                    help="apply the SGD step inside the AllReduce kernel (f2)")
-    p.add_argument("--iter-steps", type=int, default=10)
-    p.add_argument("--iter-rounds", type=int, default=3)
+    p.add_argument("--iter-steps", type=int, default=20)
+    p.add_argument("--iter-rounds", type=int, default=5)
     p.add_argument("--iter-warmup", type=int, default=2)
     p.add_argument("--iter-channels", type=int, default=4)
     p.add_argument("--iter-tree", choices=["single", "double", "rotated"], default="single")
