@@ -236,6 +236,35 @@ CCUBE_API ccube_result_t ccube_get_info(ccube_info_t *info);
  * the root. */
 CCUBE_API ccube_result_t ccube_tree_parents(int P, ccube_tree_kind_t kind, int tree, int *parent);
 
+/* Placement (reading R19; the NVSwitch form of the paper's detour routes on the
+ * DGX-1 cube mesh, §IV: with a direct path between every pair, the
+ * topology decision left is which rank hosts which tree position, root included).
+ *
+ * ccube_set_placement: tree position v of every tree is hosted by rank perm[v]
+ * for the NEXT ccube_init (host array of P ints, copied; a permutation of
+ * 0..P-1; P must equal that init's world_size).  NULL restores the identity.
+ * Children are combined in ascending rank (R2), so a placement can change fp32/
+ * bf16 results (never int32's); the oracle takes the same permutation.  Every
+ * rank must set the same placement (ccube_init checks it: INVALID_ARG).
+ * Errors: ALREADY_INITIALIZED while a communicator exists; INVALID_ARG for a
+ * non-permutation or P out of [1, CCUBE_MAX_RANKS].
+ *
+ * ccube_plan_placement (host, pure): the placement of least cost for a measured
+ * peer bandwidth matrix bw[i*P + j] (rank i -> rank j, any unit; <= 0 = no path).
+ * Every tree carries 1/T of the buffer up and down each of its edges; the cost
+ * of a placement is max over loaded directed pairs of load / bw (the slowest
+ * edge sets the pipeline's rate).  Exhaustive over P! placements, ties to the
+ * lexicographically smallest (uniform bandwidth -> identity).  Writes P ints to
+ * perm.  Errors: INVALID_ARG (NULL pointers, bad kind), UNSUPPORTED for P > 8.
+ *
+ * ccube_tree_parents_placed: ccube_tree_parents with placement perm (NULL =
+ * identity). */
+CCUBE_API ccube_result_t ccube_set_placement(const int *perm, int P);
+CCUBE_API ccube_result_t ccube_plan_placement(int P, ccube_tree_kind_t kind, const double *bw,
+                                              int *perm);
+CCUBE_API ccube_result_t ccube_tree_parents_placed(int P, ccube_tree_kind_t kind, int tree,
+                                                   const int *perm, int *parent);
+
 #ifdef __cplusplus
 }
 #endif

@@ -20,10 +20,17 @@ Rotated set (reading R17): the NVSwitch form of §IV's
 topology-aware trees — P trees, tree t = tree 0 with every rank v
 renamed (v + t) mod P, so every rank holds every tree position exactly once and
 each rank's port carries 2(P-1)/P of the buffer per direction.
+
+Placement (reading R19): the NVSwitch form of §IV's detour routes is
+the choice of which physical rank hosts which tree position.  A placement is a
+permutation perm: position v of every tree of the kind is hosted by rank
+perm[v]; children are re-listed in ascending (physical) rank, which is the
+combine order (R2), so a placement can change fp results (not int32 ones).
+Identity = the trees above.
 """
 
 from dataclasses import dataclass
-from typing import List, Tuple
+from typing import List, Optional, Sequence, Tuple
 
 
 @dataclass(frozen=True)
@@ -111,12 +118,27 @@ def rotated(P: int, t: int) -> Tree:
     return _from_parent(P, parent)
 
 
-def trees(P: int, kind: str) -> List[Tree]:
-    """kind = 'single' -> [tree0]; 'double' -> [tree0, tree1]; 'rotated' -> P trees."""
+def placed(tree: Tree, perm: Sequence[int]) -> Tree:
+    """R19: the tree with position v hosted by rank perm[v] (children re-sorted)."""
+    P = tree.P
+    if sorted(perm) != list(range(P)):
+        raise ValueError(f"placement {list(perm)} is not a permutation of 0..{P - 1}")
+    parent = [-1] * P
+    for v in range(P):
+        pv = tree.parent[v]
+        parent[perm[v]] = -1 if pv == -1 else perm[pv]
+    return _from_parent(P, parent)
+
+
+def trees(P: int, kind: str, perm: Optional[Sequence[int]] = None) -> List[Tree]:
+    """kind = 'single' -> [tree0]; 'double' -> [tree0, tree1]; 'rotated' -> P trees;
+    each placed by ``perm`` (R19) when given."""
     if kind == "single":
-        return [tree0(P)]
-    if kind == "double":
-        return [tree0(P), tree1(P)]
-    if kind == "rotated":
-        return [rotated(P, t) for t in range(max(P, 1))]
-    raise ValueError(kind)
+        ts = [tree0(P)]
+    elif kind == "double":
+        ts = [tree0(P), tree1(P)]
+    elif kind == "rotated":
+        ts = [rotated(P, t) for t in range(max(P, 1))]
+    else:
+        raise ValueError(kind)
+    return ts if perm is None else [placed(t, perm) for t in ts]

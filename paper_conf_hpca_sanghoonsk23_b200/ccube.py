@@ -9,7 +9,8 @@ Names mirror the C ABI: ``init`` (ccube_init), ``allreduce_tree`` /
 ``allreduce_tree_local``, ``gradq_set_layers``, ``gradq_wait`` /
 ``gradq_wait_local``, ``set_overlap``, ``set_channels``, ``set_threads``,
 ``set_trace``, ``register_buffers``, ``deregister_buffers``, ``finalize``,
-``last_error``, ``get_info``, ``tree_parents``.
+``last_error``, ``get_info``, ``tree_parents``, ``set_placement``,
+``plan_placement``, ``tree_parents_placed``.
 """
 
 import ctypes
@@ -41,6 +42,9 @@ EXPORTS = [
     "ccube_gradq_wait_local", "ccube_gradq_set_sgd", "ccube_set_overlap", "ccube_set_channels", "ccube_set_threads",
     "ccube_set_trace", "ccube_set_transport", "ccube_set_datapath", "ccube_finalize", "ccube_last_error", "ccube_get_info",
     "ccube_tree_parents",
+    "ccube_set_placement",
+    "ccube_plan_placement",
+    "ccube_tree_parents_placed",
 ]
 
 
@@ -101,6 +105,9 @@ def lib() -> ctypes.CDLL:
             "ccube_finalize": [],
             "ccube_get_info": [ctypes.POINTER(Info)],
             "ccube_tree_parents": [i, i, i, ctypes.POINTER(i)],
+            "ccube_set_placement": [ctypes.POINTER(i), i],
+            "ccube_plan_placement": [i, i, ctypes.POINTER(ctypes.c_double), ctypes.POINTER(i)],
+            "ccube_tree_parents_placed": [i, i, i, ctypes.POINTER(i), ctypes.POINTER(i)],
         }
         for name, args in sig.items():
             fn = getattr(L, name)
@@ -314,4 +321,32 @@ def get_info() -> dict:
 def tree_parents(P: int, kind: str, tree: int):
     out = (ctypes.c_int * P)()
     _check(lib().ccube_tree_parents(P, TREE[kind], tree, out), "ccube_tree_parents")
+    return list(out)
+
+
+def set_placement(perm: Optional[Sequence[int]]) -> None:
+    """Tree position v is hosted by rank perm[v] from the next init on (R19); None
+    restores the identity.  Every rank must pass the same permutation."""
+    if perm is None:
+        _check(lib().ccube_set_placement(None, 0), "ccube_set_placement")
+        return
+    arr = (ctypes.c_int * len(perm))(*perm)
+    _check(lib().ccube_set_placement(arr, len(perm)), "ccube_set_placement")
+
+
+def plan_placement(bw, kind: str = "double"):
+    """Least-cost placement for a P x P peer bandwidth matrix (nested sequences or
+    an array; bw[i][j] = rank i -> rank j)."""
+    P = len(bw)
+    flat = (ctypes.c_double * (P * P))(*[float(bw[i][j]) for i in range(P) for j in range(P)])
+    out = (ctypes.c_int * P)()
+    _check(lib().ccube_plan_placement(P, TREE[kind], flat, out), "ccube_plan_placement")
+    return list(out)
+
+
+def tree_parents_placed(P: int, kind: str, tree: int, perm: Optional[Sequence[int]]):
+    arr = None if perm is None else (ctypes.c_int * P)(*perm)
+    out = (ctypes.c_int * P)()
+    _check(lib().ccube_tree_parents_placed(P, TREE[kind], tree, arr, out),
+           "ccube_tree_parents_placed")
     return list(out)

@@ -714,7 +714,22 @@ struct Hello {
   int32_t world, nlocal, rank, tree_kind, device;
   uint64_t chunk_bytes;
   char busid[32];
+  int8_t place[CCUBE_MAX_RANKS];  // the placement (R19), identity when none was set
 };
+
+// Placement set by ccube_set_placement for the next ccube_init (0 = identity).  Lives
+// outside Comm: it is configuration, kept across finalize/init.
+int g_place[CCUBE_MAX_RANKS];
+int g_place_P = 0;
+
+bool is_permutation(const int *perm, int P) {
+  bool seen[CCUBE_MAX_RANKS] = {};
+  for (int v = 0; v < P; ++v) {
+    if (perm[v] < 0 || perm[v] >= P || seen[perm[v]]) return false;
+    seen[perm[v]] = true;
+  }
+  return true;
+}
 
 }  // namespace
 }  // namespace ccube
@@ -743,6 +758,9 @@ ccube_result_t ccube_init(const ccube_world_t *world, ccube_tree_kind_t tree_kin
     return fail(CCUBE_ERR_INVALID_ARG, "bad tree kind %d", (int)tree_kind);
   if (world->nlocal < P && !world->allgather)
     return fail(CCUBE_ERR_INVALID_ARG, "allgather callback required when nlocal < world_size");
+  if (g_place_P != 0 && g_place_P != P)
+    return fail(CCUBE_ERR_INVALID_ARG, "the placement was set for %d ranks, world_size is %d",
+                g_place_P, P);
   if (chunk_bytes == 0) chunk_bytes = CCUBE_DEFAULT_CHUNK_BYTES;
   int channels = env_int("CCUBE_CHANNELS", 0);
   if (channels < 0 || channels > CCUBE_MAX_CHANNELS)
@@ -780,7 +798,10 @@ ccube_result_t ccube_init(const ccube_world_t *world, ccube_tree_kind_t tree_kin
   g.sys_scope = g.nproc > 1;
   g.timeout_ns = static_cast<uint64_t>(env_int("CCUBE_WATCHDOG_MS", 10000)) * 1000000ull;
   g.use_memop = env_int("CCUBE_GATE_KERNEL", 0) == 0;
-  for (int t = 0; t < g.ntrees; ++t) build_tree(P, tree_kind, t, &g.trees[t]);
+  for (int t = 0; t < g.ntrees; ++t) {
+    build_tree(P, tree_kind, t, &g.trees[t]);
+    if (g_place_P == P) place_tree(g_place, &g.trees[t]);
+  }
 
   // (i) config agreement — host only, so it also runs (and can be tested) without a GPU
   Hello mine;
@@ -792,6 +813,7 @@ ccube_result_t ccube_init(const ccube_world_t *world, ccube_tree_kind_t tree_kin
   mine.tree_kind = tree_kind;
   mine.device = g.device;
   mine.chunk_bytes = chunk_bytes;
+  for (int v = 0; v < P; ++v) mine.place[v] = static_cast<int8_t>(g_place_P == P ? g_place[v] : v);
   if (cudaDeviceGetPCIBusId(mine.busid, sizeof mine.busid, g.device) != cudaSuccess)
     snprintf(mine.busid, sizeof mine.busid, "nodevice-%d", g.rank0);
   std::vector<Hello> all(g.nproc);
@@ -805,11 +827,11 @@ ccube_result_t ccube_init(const ccube_world_t *world, ccube_tree_kind_t tree_kin
     const Hello &h = all[p];
     if (h.magic != mine.magic || h.world != P || h.nlocal != g.nlocal ||
         h.rank != p * g.nlocal || h.tree_kind != mine.tree_kind ||
-        h.chunk_bytes != mine.chunk_bytes) {
+        h.chunk_bytes != mine.chunk_bytes || memcmp(h.place, mine.place, sizeof h.place)) {
       g = Comm();
       return fail(CCUBE_ERR_INVALID_ARG,
                   "ranks disagree on the configuration (process %d: world %d nlocal %d rank %d "
-                  "tree %d chunk %llu)",
+                  "tree %d chunk %llu, or the placement)",
                   p, h.world, h.nlocal, h.rank, h.tree_kind, (unsigned long long)h.chunk_bytes);
     }
     // Several processes on one GPU only time-slice (no MPS): their spinning kernels
@@ -1067,6 +1089,47 @@ ccube_result_t ccube_get_info(ccube_info_t *info) {
   info->last_ctas = g.last_ctas;
   info->datapath = g.datapath;
   info->last_tma = g.last_tma;
+  return CCUBE_SUCCESS;
+}
+
+ccube_result_t ccube_set_placement(const int *perm, int P) {
+  std::lock_guard<std::mutex> lk(g_mu);
+  if (g.init) return fail(CCUBE_ERR_ALREADY_INITIALIZED, "set the placement before ccube_init");
+  if (!perm) {
+    g_place_P = 0;
+    return CCUBE_SUCCESS;
+  }
+  if (P < 1 || P > CCUBE_MAX_RANKS) return fail(CCUBE_ERR_INVALID_ARG, "bad P %d", P);
+  if (!is_permutation(perm, P))
+    return fail(CCUBE_ERR_INVALID_ARG, "placement is not a permutation of 0..%d", P - 1);
+  for (int v = 0; v < P; ++v) g_place[v] = perm[v];
+  g_place_P = P;
+  return CCUBE_SUCCESS;
+}
+
+ccube_result_t ccube_plan_placement(int P, ccube_tree_kind_t kind, const double *bw, int *perm) {
+  if (P < 1 || P > CCUBE_MAX_RANKS || !bw || !perm)
+    return fail(CCUBE_ERR_INVALID_ARG, "bad P, bw or perm");
+  if (kind != CCUBE_TREE_SINGLE && kind != CCUBE_TREE_DOUBLE && kind != CCUBE_TREE_ROTATED)
+    return fail(CCUBE_ERR_INVALID_ARG, "bad tree kind %d", (int)kind);
+  if (!plan_placement(P, kind, bw, perm))
+    return fail(CCUBE_ERR_UNSUPPORTED, "placement planning supports P <= 8");
+  return CCUBE_SUCCESS;
+}
+
+ccube_result_t ccube_tree_parents_placed(int P, ccube_tree_kind_t kind, int tree,
+                                         const int *perm, int *parent) {
+  if (P < 1 || P > kTreeMaxP || !parent) return fail(CCUBE_ERR_INVALID_ARG, "bad P or parent");
+  if (kind != CCUBE_TREE_SINGLE && kind != CCUBE_TREE_DOUBLE && kind != CCUBE_TREE_ROTATED)
+    return fail(CCUBE_ERR_INVALID_ARG, "bad tree kind %d", (int)kind);
+  if (tree < 0 || tree >= num_trees(P, kind))
+    return fail(CCUBE_ERR_INVALID_ARG, "bad tree index %d", tree);
+  if (perm && (P > CCUBE_MAX_RANKS || !is_permutation(perm, P)))
+    return fail(CCUBE_ERR_INVALID_ARG, "placement is not a permutation of 0..%d", P - 1);
+  Tree t;
+  build_tree(P, kind, tree, &t);
+  if (perm) place_tree(perm, &t);
+  for (int v = 0; v < P; ++v) parent[v] = t.parent[v];
   return CCUBE_SUCCESS;
 }
 

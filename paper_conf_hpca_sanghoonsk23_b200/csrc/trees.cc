@@ -13,6 +13,9 @@
 // two agree for every P.
 #include "trees.h"
 
+#include <algorithm>
+#include <limits>
+
 namespace ccube {
 
 namespace {
@@ -75,6 +78,57 @@ void build_tree(int P, int kind, int which, Tree *out) {
     const int p = out->parent[c];
     if (p >= 0) out->child[p][out->nchild[p]++] = c;
   }
+}
+
+void place_tree(const int *perm, Tree *t) {
+  const int P = t->P;
+  int parent[kTreeMaxP];
+  for (int v = 0; v < P; ++v)
+    parent[perm[v]] = t->parent[v] < 0 ? -1 : perm[t->parent[v]];
+  for (int v = 0; v < P; ++v) {
+    t->parent[v] = parent[v];
+    t->nchild[v] = 0;
+    if (parent[v] < 0) t->root = v;
+  }
+  for (int c = 0; c < P; ++c)  // ascending rank
+    if (parent[c] >= 0) t->child[parent[c]][t->nchild[parent[c]]++] = c;
+}
+
+bool plan_placement(int P, int kind, const double *bw, int *perm) {
+  if (P < 1 || P > 8) return false;
+  // directed edge loads of the identity placement, in units of 1/T of the buffer
+  int load[8][8] = {};
+  const int T = num_trees(P, kind);
+  for (int t = 0; t < T; ++t) {
+    Tree tr;
+    build_tree(P, kind, t, &tr);
+    for (int c = 0; c < P; ++c) {
+      if (tr.parent[c] < 0) continue;
+      ++load[c][tr.parent[c]];
+      ++load[tr.parent[c]][c];
+    }
+  }
+  int p[8];
+  for (int v = 0; v < P; ++v) p[v] = perm[v] = v;
+  double best = std::numeric_limits<double>::infinity();
+  bool first = true;
+  do {  // lexicographic order from the identity; strict improvement only
+    double cost = 0.0;
+    for (int i = 0; i < P; ++i)
+      for (int j = 0; j < P; ++j) {
+        if (!load[i][j]) continue;
+        const double b = bw[p[i] * P + p[j]];
+        const double c = b > 0 ? (static_cast<double>(load[i][j]) / T) / b
+                               : std::numeric_limits<double>::infinity();
+        cost = std::max(cost, c);
+      }
+    if (first || cost < best) {
+      best = cost;
+      first = false;
+      for (int v = 0; v < P; ++v) perm[v] = p[v];
+    }
+  } while (std::next_permutation(p, p + P));
+  return true;
 }
 
 int child_slot(const Tree &t, int parent, int c) {

@@ -472,3 +472,67 @@ def test_parity_task_order(comm, monkeypatch, order, kind, sgd):
         for w in ws:
             np.testing.assert_array_equal(to_numpy(w, "float32"), want)
         ccube.gradq_set_sgd(None)
+
+
+# ---- placement (reading R19) ---------------------------------------------------------
+def _placed_run(P, kind, dtype, perm, count, chunk, channels=3, overlap=True, seed=21, xs=None):
+    ccube.set_placement(perm)
+    try:
+        ccube.init_loopback(P, kind, chunk)
+        try:
+            ccube.set_channels(channels)
+            ccube.set_overlap(overlap)
+            if xs is None:
+                xs = [inputs.gradients(r, count, dtype, seed=seed) for r in range(P)]
+            ts = [to_torch(x, dtype).cuda() for x in xs]
+            ccube.allreduce_tree_local(ts)
+            torch.cuda.synchronize()
+            return xs, [to_numpy(t, dtype) for t in ts]
+        finally:
+            ccube.finalize()
+    finally:
+        ccube.set_placement(None)
+
+
+@pytest.mark.parametrize("P", [3, 4, 8])
+@pytest.mark.parametrize("kind", ["single", "double", "rotated"])
+@pytest.mark.parametrize("dtype", ["int32", "float32", "bfloat16"])
+@pytest.mark.parametrize("overlap", [True, False])
+def test_parity_placement(P, kind, dtype, overlap):
+    """A placed tree set (position v on rank perm[v]) is bit-exact to the oracle
+    with the same permutation; ragged tail, several chunks per tree."""
+    perm = [int(v) for v in np.random.default_rng(P + 7).permutation(P)]
+    chunk = 4096
+    count = 9 * (chunk // 4) + 5
+    xs, outs = _placed_run(P, kind, dtype, perm, count, chunk, overlap=overlap)
+    ref = oar.reference(xs, kind, chunk, dtype, perm=perm)[0]
+    for r in range(P):
+        assert np.array_equal(outs[r].view(np.uint8), ref.view(np.uint8)), f"rank {r}"
+
+
+def test_placement_order_pin_gpu():
+    """The hand-derived pin of tests/test_placement.py on the GPU: identity 1.0,
+    reversal 0.0 for x = (1, 2^24, 1, -2^24)."""
+    xs = [np.array([v] * 4, np.float32) for v in (1.0, 2.0 ** 24, 1.0, -2.0 ** 24)]
+    _, outs = _placed_run(4, "single", "float32", [0, 1, 2, 3], 4, 16, channels=1, xs=xs)
+    assert all(o[0] == 1.0 for o in outs)
+    _, outs = _placed_run(4, "single", "float32", [3, 2, 1, 0], 4, 16, channels=1, xs=xs)
+    assert all(o[0] == 0.0 for o in outs)
+
+
+def test_parity_placement_full_size_resnet50():
+    """ResNet-50 gradient set, P = 8, double tree, a planned placement for a matrix
+    with two slow pairs, bench launch configuration (auto channels)."""
+    from oracle import placement as opl
+    P = 8
+    bw = np.full((P, P), 100.0)
+    bw[0, 4] = bw[4, 0] = bw[3, 7] = bw[7, 3] = 10.0
+    perm = ccube.plan_placement(bw, "double")
+    assert perm == opl.plan(P, "double", bw) and perm != list(range(P))
+    ends = workloads.layer_ends("resnet50")
+    count = ends[-1]
+    xs = [inputs.gradients(r, count, "float32", layer_ends=ends) for r in range(P)]
+    _, outs = _placed_run(P, "double", "float32", perm, count, 256 << 10, channels=0, xs=xs)
+    ref = oar.reference(xs, "double", 256 << 10, "float32", perm=perm)[0]
+    for r in range(P):
+        assert np.array_equal(outs[r], ref), f"rank {r}"
