@@ -56,6 +56,8 @@ def parse():
     p.add_argument("--no-nccl", action="store_true",
                    help="N>1: skip the NCCL Ring/Tree/default comparison on the same buffer")
     p.add_argument("--nccl-steps", type=int, default=20)
+    p.add_argument("--plan-placement", action="store_true",
+                   help="N>1: measure peer bandwidth and place the trees on it (R19)")
     p.add_argument("--cpu-seconds", type=float, default=10.0,
                    help="cpu_baseline: repeat the oracle sample until this much CPU work")
     p.add_argument("--cpu-sample-chunks", type=int, default=0,
@@ -259,6 +261,12 @@ def run_ccube(a):
     pristine = [h.to(dev) for h in host]
     bufs = [p.clone() for p in pristine]
 
+    placement_info = None
+    if multi and a.plan_placement:   # R19: measured peer bandwidth -> tree placement
+        from paper_conf_hpca_sanghoonsk23_b200 import placement
+        perm, pbw = placement.plan(dist.group.WORLD, kind=a.tree)
+        ccube.set_placement(perm)
+        placement_info = {"perm": perm, "peer_gbs": pbw}
     if multi:
         ccube.init_distributed(dist.group.WORLD, tree=a.tree, chunk_bytes=a.chunk_bytes)
     else:
@@ -441,6 +449,8 @@ def run_ccube(a):
         }
         if nccl is not None:
             line["nccl"] = nccl
+        if placement_info is not None:
+            line["placement"] = placement_info
         print(json.dumps(line), flush=True)
     if multi:
         dist.destroy_process_group()
