@@ -23,7 +23,7 @@ def _free_port():
     return p
 
 
-def _worker(rank, world, port, kind, dtype, count, chunk, q):
+def _worker(rank, world, port, kind, dtype, count, chunk, q, perm=None):
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)
     os.environ["CCUBE_ALLOW_SHARED_GPU"] = "1"
@@ -33,6 +33,7 @@ def _worker(rank, world, port, kind, dtype, count, chunk, q):
     try:
         torch.cuda.set_device(0)
         dist.init_process_group("gloo", rank=rank, world_size=world)
+        ccube.set_placement(perm)
         ccube.init_distributed(dist.group.WORLD, tree=kind, chunk_bytes=chunk)
         ccube.set_channels(2)
         x = inputs.gradients(rank, count, dtype)
@@ -68,12 +69,12 @@ def _worker(rank, world, port, kind, dtype, count, chunk, q):
             dist.destroy_process_group()
 
 
-def _run(world, kind, dtype, count, chunk):
+def _run(world, kind, dtype, count, chunk, perm=None):
     import torch.multiprocessing as mp
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_worker, args=(r, world, port, kind, dtype, count, chunk, q))
+    procs = [ctx.Process(target=_worker, args=(r, world, port, kind, dtype, count, chunk, q, perm))
              for r in range(world)]
     for p in procs:
         p.start()
@@ -95,6 +96,23 @@ def test_multiprocess_ipc_parity(world, kind, dtype):
     res = _run(world, kind, dtype, count, chunk)
     xs = [inputs.gradients(r, count, dtype) for r in range(world)]
     ref = oar.reference(xs, kind, chunk, dtype)[0]
+    for rank, err, out, early in res:
+        assert err == "", f"rank {rank}: {err}"
+        assert np.array_equal(out, ref), f"rank {rank} differs from the oracle"
+        assert not early, f"rank {rank}: a gate opened before its layer landed"
+
+
+def test_multiprocess_ipc_parity_placed():
+    """A placed double tree (R19) across processes: bit-exact to the oracle with the
+    same permutation (the gradient-queue gates included)."""
+    from oracle import allreduce as oar
+    from paper_conf_hpca_sanghoonsk23_b200 import inputs
+    world, kind, dtype, perm = 4, "double", "float32", [2, 0, 3, 1]
+    count, chunk = 50_001, 16 << 10
+    res = _run(world, kind, dtype, count, chunk, perm)
+    xs = [inputs.gradients(r, count, dtype) for r in range(world)]
+    ref = oar.reference(xs, kind, chunk, dtype, perm=perm)[0]
+    assert not np.array_equal(ref, oar.reference(xs, kind, chunk, dtype)[0])
     for rank, err, out, early in res:
         assert err == "", f"rank {rank}: {err}"
         assert np.array_equal(out, ref), f"rank {rank} differs from the oracle"
