@@ -56,6 +56,8 @@ def parse():
     p.add_argument("--no-nccl", action="store_true",
                    help="N>1: skip the NCCL Ring/Tree/default comparison on the same buffer")
     p.add_argument("--nccl-steps", type=int, default=20)
+    p.add_argument("--max-elems", type=int, default=0,
+                   help="test runs only: time a prefix of the workload (0 = all of it)")
     p.add_argument("--plan-placement", action="store_true",
                    help="N>1: measure peer bandwidth and place the trees on it (R19)")
     p.add_argument("--cpu-seconds", type=float, default=10.0,
@@ -232,14 +234,22 @@ def run_ccube(a):
     rank = int(os.environ.get("RANK", "0"))
     local_rank = int(os.environ.get("LOCAL_RANK", "0"))
     multi = world > 1
-    torch.cuda.set_device(local_rank if multi else 0)
+    # test mode for the N>1 path on a one-GPU box: every rank on cuda:0 (with
+    # CCUBE_ALLOW_SHARED_GPU=1), gloo for the host plumbing, no NCCL comparison
+    shared = multi and os.environ.get("CCUBE_BENCH_SHARED_GPU") == "1"
+    torch.cuda.set_device(local_rank if multi and not shared else 0)
     dev = torch.device("cuda", torch.cuda.current_device())
     if multi:
-        dist.init_process_group("nccl", device_id=dev)
+        if shared:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=dev)
     P = world if multi else a.ranks
     nloc = 1 if multi else P
 
     ends = workloads.layer_ends(a.workload)
+    if a.max_elems:   # test runs only: a prefix of the workload
+        ends = [min(e, a.max_elems) for e in ends]
     count = ends[-1]
     tdt = {"float32": torch.float32, "bfloat16": torch.bfloat16, "int32": torch.int32}[a.dtype]
     es = torch.tensor([], dtype=tdt).element_size()
@@ -315,9 +325,7 @@ def run_ccube(a):
     ms = [s.elapsed_time(e) for s, e in evs]
     total_ms = float(np.sum(ms))
     if multi:
-        t = torch.tensor([total_ms], device=dev)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        total_ms = t.item()
+        total_ms = _allmax(total_ms, None if shared else dev)
     clk = clocks.stop()
     ms_step = total_ms / a.steps
     bw, alg = busbw(nbytes, ms_step / 1e3, P)
@@ -373,9 +381,7 @@ def run_ccube(a):
         torch.cuda.synchronize()
         e2e_ms = e0.elapsed_time(e1) / a.e2e_steps
         if multi:
-            t = torch.tensor([e2e_ms], device=dev)
-            dist.all_reduce(t, op=dist.ReduceOp.MAX)
-            e2e_ms = t.item()
+            e2e_ms = _allmax(e2e_ms, None if shared else dev)
         ebw, _ = busbw(nbytes, e2e_ms / 1e3, P)
         ok_e2e = all(torch.equal(o, outs[0]) for o in outs[1:]) if not multi else None
         e2e = {"value": ebw, "unit": "GB/s", "ms_per_step": e2e_ms,
@@ -416,7 +422,7 @@ def run_ccube(a):
 
     # ---- NCCL on the same box and buffer (the comparison baseline, N>1 only)
     nccl = None
-    if multi and not a.no_nccl:
+    if multi and not a.no_nccl and not shared:
         nccl = nccl_compare(a, dev, bufs[0], pristine[0], nbytes, P, stream)
 
     info = ccube.get_info()
@@ -583,6 +589,15 @@ def run_iteration(a, P, log=None):
     out["exposed_cut_C2_vs_B"] = cut("C2", "B")      # chaining alone
     out["exposed_cut_CC_vs_C1"] = cut("CC", "C1")    # chaining on top of the overlapped tree
     return out
+
+
+def _allmax(x, dev):
+    """Max over ranks of a host float (on ``dev`` for NCCL, on the host for gloo)."""
+    import torch
+    import torch.distributed as dist
+    t = torch.tensor([float(x)], dtype=torch.float64, device=dev)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return t.item()
 
 
 def nccl_compare(a, dev, buf, pristine, nbytes, P, stream):
