@@ -536,3 +536,37 @@ def test_parity_placement_full_size_resnet50():
     ref = oar.reference(xs, "double", 256 << 10, "float32", perm=perm)[0]
     for r in range(P):
         assert np.array_equal(outs[r], ref), f"rank {r}"
+
+
+@pytest.mark.parametrize("kind", ["single", "double"])
+def test_max_size_1gib_ragged(comm, kind):
+    """configs[4]'s largest message (1 GiB per rank, fp32) minus a ragged tail of 37
+    elements, P = 8, 256 KiB chunks (K = 4096). Each rank's buffer is its seeded
+    generator block of B = 2^20 + 7 elements repeated (B is not a multiple of the chunk,
+    so no two chunks see the same data); sampled chunks bit-exact vs the oracle's fold
+    on the same values (first, the ragged last, random), every rank identical."""
+    from oracle import trees as otrees
+
+    P, chunk, B = 8, 256 << 10, (1 << 20) + 7
+    count = (1 << 28) - 37
+    comm(P, kind, chunk)
+    base = [inputs.gradients(r, B, "float32", seed=11) for r in range(P)]
+    ts = []
+    for r in range(P):
+        b = torch.from_numpy(base[r]).cuda()
+        ts.append(b.repeat((count + B - 1) // B)[:count].contiguous())
+    ccube.allreduce_tree_local(ts)
+    torch.cuda.synchronize()
+    K = partition.num_chunks(count, chunk, 4)
+    assert K == 4096
+    trees = otrees.trees(P, kind)
+    rng = np.random.default_rng(1)
+    for c in sorted({0, 1, K - 2, K - 1, *rng.integers(0, K, 6).tolist()}):
+        lo, hi = partition.chunk_range(c, count, chunk, 4)
+        idx = np.arange(lo, hi) % B
+        tree = trees[partition.tree_of_chunk(c, len(trees))]
+        want = oar.fold([x[idx] for x in base], tree, tree.root, "float32")
+        for r in (0, 7):
+            assert np.array_equal(to_numpy(ts[r][lo:hi], "float32"), want), (c, r)
+    for r in range(1, P):
+        assert torch.equal(ts[r], ts[0])
