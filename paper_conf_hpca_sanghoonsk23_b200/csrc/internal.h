@@ -108,6 +108,7 @@ struct LaunchArgs {
   int tma;                    // datapath: 0 = register-staged LSU, 1 = TMA bulk-load ring
   int elem_size;              // bytes per element (2 or 4)
   int split_control;          // 1 = separate poll and publish warps (warps 0, 1)
+  int backoff_ns;             // data warps' readiness-spin back-off (0 = spin)
 };
 
 // Kernel launcher (tree_allreduce.cu).  Returns a cudaError_t as int.

@@ -169,6 +169,7 @@ struct Comm {
   int datapath = CCUBE_DATAPATH_AUTO;  // CCUBE_DATAPATH env / ccube_set_datapath
   int last_tma = 0;
   int split_control = 1;              // CCUBE_SPLIT_CONTROL env: poll and publish warps
+  int backoff_ns = 64;                // CCUBE_BACKOFF_NS env: data warps' spin back-off
   int task_order = 0;                 // CCUBE_TASK_ORDER env: block -> task placement
   bool sgd = false;                 // fused SGD update (f2)
   float sgd_alpha = 0.0f;
@@ -601,6 +602,7 @@ ccube_result_t allreduce_impl(void *const *bufs, size_t count, ccube_dtype_t dty
   a.sgd_alpha = g.sgd_alpha;
   a.tma = tma;
   a.split_control = g.split_control;
+  a.backoff_ns = g.backoff_ns;
   a.elem_size = static_cast<int>(es);
   a.params = R->d_params;
 
@@ -792,6 +794,7 @@ ccube_result_t ccube_init(const ccube_world_t *world, ccube_tree_kind_t tree_kin
   g.l2_hints = env_int("CCUBE_L2_HINTS", 1);
   g.split_control = env_int("CCUBE_SPLIT_CONTROL", 1) != 0 ? 1 : 0;
   g.task_order = env_int("CCUBE_TASK_ORDER", 0);
+  g.backoff_ns = env_int("CCUBE_BACKOFF_NS", 64);
   g.datapath = env_int("CCUBE_DATAPATH", CCUBE_DATAPATH_AUTO);
   if (g.datapath != CCUBE_DATAPATH_LSU && g.datapath != CCUBE_DATAPATH_TMA)
     g.datapath = CCUBE_DATAPATH_AUTO;

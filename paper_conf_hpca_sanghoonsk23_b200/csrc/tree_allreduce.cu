@@ -734,7 +734,7 @@ __device__ void lsu_stream(const LaunchArgs &a, const Endpoints &e, int t, int j
       if (lane == 0) {  // upstream not there yet: back off so busy warps get the issue slots
         while ((r = ld_acquire_cta(&sh.ready)) <= k &&
                !*reinterpret_cast<volatile int *>(&sh.abort))
-          __nanosleep(64);
+          if (a.backoff_ns > 0) __nanosleep(a.backoff_ns);
       }
       r = __shfl_sync(0xffffffffu, r, 0);
       if (r <= k) return;  // aborted
