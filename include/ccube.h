@@ -110,8 +110,16 @@ typedef struct {
  * IPC over NVLink/NVSwitch when nlocal == 1) and zeroes the monotone counters.
  *   chunk_bytes: bytes per pipelined chunk ("the amount of data that is
  *     communicated between neighboring nodes in each step", fn3 P:L88); 0 selects
- *     CCUBE_DEFAULT_CHUNK_BYTES.  Must be a multiple of 16 * channels.
- * Errors: INVALID_ARG (bad world/tree/chunk, ranks disagree on the config),
+ *     CCUBE_DEFAULT_CHUNK_BYTES.  Must be a positive multiple of 16 (channel
+ *     slices are whole 2 KB units; a chunk shorter than J units leaves the extra
+ *     channels an empty slice).
+ *   The launch settings read from the environment (CCUBE_CHANNELS, CCUBE_THREADS,
+ *   CCUBE_DATAPATH, CCUBE_TRANSPORT, CCUBE_L2_HINTS, CCUBE_SPLIT_CONTROL) are part of
+ *   the configuration every rank must share; ccube_init checks them.
+ *   With several processes every tree neighbour on another GPU must be a CUDA peer
+ *   (cudaDeviceCanAccessPeer), checked collectively. 
+ * Errors: INVALID_ARG (bad world/tree/chunk, ranks disagree on the config or the
+ * launch settings),
  * ALREADY_INITIALIZED, UNSUPPORTED (world_size > CCUBE_MAX_RANKS, two processes on
  * one GPU, no peer access), BOOTSTRAP (allgather callback failed), CUDA. */
 CCUBE_API ccube_result_t ccube_init(const ccube_world_t *world, ccube_tree_kind_t tree_kind,
@@ -179,10 +187,20 @@ CCUBE_API ccube_result_t ccube_gradq_set_sgd(void *const *weights, size_t bytes,
  * the paper's baseline "B").  Values are bitwise identical. */
 CCUBE_API ccube_result_t ccube_set_overlap(int on);
 
-/* Channels J per tree (CTA slices of every chunk); all ranks must agree.  0 = auto
- * (CCUBE_CHANNELS env, else the most channels whose CTAs are co-resident, capped at
- * one channel per two 2 KB units of a chunk, or per unit for buffers of >= 16 chunks).  `threads` = data threads per CTA (32..256,
- * multiple of 32; CCUBE_THREADS env, default 256); each CTA adds one control warp. */
+/* Settings every rank must share (set_overlap above, set_channels, set_threads,
+ * set_datapath, set_transport, gradq_set_sgd on/off): with several processes these
+ * setters are COLLECTIVE — every rank calls them in the same order, the value is
+ * checked through the allgather callback, and every rank returns INVALID_ARG if
+ * any rank passed a different (or invalid) value, leaving the old setting in place.
+ *
+ * Channels J per tree (CTA slices of every chunk).  0 = auto (CCUBE_CHANNELS env,
+ * else the most channels whose CTAs are co-resident on EVERY process — the task
+ * count is the maximum over all processes, which depends on every rank's role in
+ * every tree, and the capacity the minimum over GPUs — capped at one channel per
+ * two 2 KB units of a chunk, or per unit for buffers of >= 16 chunks).  Both ends of
+ * an edge therefore always slice chunks alike.  `threads` = data threads per CTA
+ * (32..256, multiple of 32; CCUBE_THREADS env, default 256); each CTA adds two
+ * control warps. */
 CCUBE_API ccube_result_t ccube_set_channels(int channels);
 CCUBE_API ccube_result_t ccube_set_threads(int threads);
 
@@ -214,6 +232,44 @@ CCUBE_API ccube_result_t ccube_set_transport(int mode);
  * stores %globaltimer (ns) into trace[((r * ntrees + t) * kmax + k) * J + j].
  * NULL disables.  Device pointer of nlocal*ntrees*kmax*J uint64. */
 CCUBE_API ccube_result_t ccube_set_trace(uint64_t *trace, size_t kmax);
+
+/* ccube_barrier — collective, device-side: enqueue on `stream` a barrier across all
+ * ranks over tree 0's edges (arrive up to the root, release down), using the same
+ * monotone counters as the AllReduce; no host synchronisation.  Work enqueued on
+ * `stream` after it starts only after every rank has reached it (bench.py puts it
+ * before the start event of every timed step).  A no-op when one
+ * process hosts every rank (stream order already orders the launch).  Errors:
+ * NOT_INITIALIZED, TIMEOUT (an earlier watchdog abort), CUDA. */
+CCUBE_API ccube_result_t ccube_barrier(void *stream);
+
+/* ccube_measure_peer_bandwidth — collective (one process per GPU, after
+ * ccube_init): the NVLink roofline instrument (SURVEY §8(d) "P2P port-peak
+ * microbenchmark").  Times, on the device and after a ccube_barrier, the
+ * AllReduce's own cross-GPU data path — 128-bit loads from local HBM, 128-bit
+ * stores into a peer's HBM — for `bytes` per destination, best of `iters`.
+ *   pair_gbs[i * P + j]: GB/s of rank i's stores into rank j while every rank
+ *     stores to its k-th successor at once (k = (j - i) mod P; every port carries one
+ *     stream per direction); 0 on the diagonal.
+ *   fanout_gbs[m], m = 1..P-1: per-GPU egress GB/s (minimum over ranks) while every
+ *     rank stores to its m successors at once; fanout_gbs[0] = 0.
+ *   Host arrays of P * P and P doubles, identical on every rank on return.  The
+ *   library allocates (and frees) `bytes` + P * `bytes` of scratch and maps every
+ *   peer's scratch (not only tree neighbours).
+ * Errors: NOT_INITIALIZED; UNSUPPORTED unless nlocal == 1 and world_size >= 2;
+ * INVALID_ARG (bytes not a positive multiple of 16, iters < 1, NULL); CUDA. */
+CCUBE_API ccube_result_t ccube_measure_peer_bandwidth(size_t bytes, int iters, double *pair_gbs,
+                                                      double *fanout_gbs);
+
+/* ccube_plan_launch (host, pure) — the launch geometry the library uses for a call
+ * of `bytes` per rank with `channels` (0 = auto) and overlap (1 = C1, 0 = B) when
+ * every GPU can hold `cap_ctas` co-resident CTAs: writes the channel count J, the
+ * CTAs of the process hosting `rank` (nlocal ranks per process, AUTO transport, no
+ * fused update) and the maximum over all processes.  J never depends on `rank`
+ * (SURVEY §8(a3)); tests check that for every rank.  Errors: INVALID_ARG. */
+CCUBE_API ccube_result_t ccube_plan_launch(int P, ccube_tree_kind_t kind, int nlocal, int rank,
+                                           size_t bytes, size_t chunk_bytes, int overlap,
+                                           int channels, int cap_ctas, int *channels_out,
+                                           int *ctas_out, int *max_ctas_out);
 
 CCUBE_API ccube_result_t ccube_finalize(void);
 

@@ -23,7 +23,7 @@ INCLUDE = os.path.join(ROOT, "include")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 NVCC_FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-fvisibility=hidden",
               "-Xptxas", "-v", "--expt-relaxed-constexpr"]
-SOURCES = ["tree_allreduce.cu", "runtime.cc", "trees.cc"]
+SOURCES = ["tree_allreduce.cu", "runtime.cc", "trees.cc", "plan.cc"]
 
 
 def nvcc() -> str:

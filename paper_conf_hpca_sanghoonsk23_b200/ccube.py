@@ -8,9 +8,9 @@ call raises — there is no CPU fallback.
 Names mirror the C ABI: ``init`` (ccube_init), ``allreduce_tree`` /
 ``allreduce_tree_local``, ``gradq_set_layers``, ``gradq_wait`` /
 ``gradq_wait_local``, ``set_overlap``, ``set_channels``, ``set_threads``,
-``set_trace``, ``register_buffers``, ``deregister_buffers``, ``finalize``,
+``set_trace``, ``register_buffers``, ``deregister_buffers``, ``barrier``, ``finalize``,
 ``last_error``, ``get_info``, ``tree_parents``, ``set_placement``,
-``plan_placement``, ``tree_parents_placed``.
+``plan_placement``, ``tree_parents_placed``, ``plan_launch``.
 """
 
 import ctypes
@@ -45,6 +45,9 @@ EXPORTS = [
     "ccube_set_placement",
     "ccube_plan_placement",
     "ccube_tree_parents_placed",
+    "ccube_barrier",
+    "ccube_plan_launch",
+    "ccube_measure_peer_bandwidth",
 ]
 
 
@@ -108,6 +111,11 @@ def lib() -> ctypes.CDLL:
             "ccube_set_placement": [ctypes.POINTER(i), i],
             "ccube_plan_placement": [i, i, ctypes.POINTER(ctypes.c_double), ctypes.POINTER(i)],
             "ccube_tree_parents_placed": [i, i, i, ctypes.POINTER(i), ctypes.POINTER(i)],
+            "ccube_barrier": [vp],
+            "ccube_plan_launch": [i, i, i, i, sz, sz, i, i, i, ctypes.POINTER(i),
+                                  ctypes.POINTER(i), ctypes.POINTER(i)],
+            "ccube_measure_peer_bandwidth": [sz, i, ctypes.POINTER(ctypes.c_double),
+                                             ctypes.POINTER(ctypes.c_double)],
         }
         for name, args in sig.items():
             fn = getattr(L, name)
@@ -247,6 +255,32 @@ def allreduce_tree_local_ptrs(ptrs: Sequence[int], count: int, dtype: str, strea
     _check(lib().ccube_allreduce_tree_local(_ptr_array(list(ptrs)), count, DTYPE[dtype],
                                             _stream_handle(stream)),
            "ccube_allreduce_tree_local")
+
+
+def barrier(stream=None) -> None:
+    """ccube_barrier: device-side barrier across all ranks, enqueued on ``stream``."""
+    _check(lib().ccube_barrier(_stream_handle(stream)), "ccube_barrier")
+
+
+def plan_launch(P: int, kind: str, nlocal: int, rank: int, nbytes: int, chunk_bytes: int = 0,
+                overlap: bool = True, channels: int = 0, cap_ctas: int = 296):
+    """ccube_plan_launch (host only): (J, CTAs of rank's process, max CTAs over processes)."""
+    j, n, m = ctypes.c_int(), ctypes.c_int(), ctypes.c_int()
+    _check(lib().ccube_plan_launch(P, TREE[kind], nlocal, rank, nbytes, chunk_bytes,
+                                   1 if overlap else 0, channels, cap_ctas, ctypes.byref(j),
+                                   ctypes.byref(n), ctypes.byref(m)), "ccube_plan_launch")
+    return j.value, n.value, m.value
+
+
+def measure_peer_bandwidth(nbytes: int = 64 << 20, iters: int = 5):
+    """ccube_measure_peer_bandwidth (collective, one process per GPU): returns
+    (pair GB/s as a P x P list, per-GPU egress GB/s for fan-out m = 0..P-1)."""
+    P = get_info()["world_size"]
+    pair = (ctypes.c_double * (P * P))()
+    fan = (ctypes.c_double * P)()
+    _check(lib().ccube_measure_peer_bandwidth(nbytes, iters, pair, fan),
+           "ccube_measure_peer_bandwidth")
+    return [[pair[i * P + j] for j in range(P)] for i in range(P)], list(fan)
 
 
 # ------------------------------------------------------------------ gradient queue

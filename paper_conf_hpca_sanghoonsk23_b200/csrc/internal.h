@@ -41,6 +41,13 @@ CCUBE_HD inline size_t flag_offset(int tree, int kind, int ch) {
 constexpr size_t kFlagBytes =
     static_cast<size_t>(kMaxTrees) * kNumFlagKinds * kMaxChannels * kFlagStride;
 
+// Device-side barrier (ccube_barrier) over tree 0's edges, after the counters:
+// "arrive" written by child slot s into its parent, "release" written by the parent
+// into the child; single-writer monotone u64 like every other counter.
+enum BarrierSlot { kBarArrive0 = 0, kBarArrive1 = 1, kBarRelease = 2, kBarSlots = 3 };
+CCUBE_HD inline size_t barrier_offset(int slot) { return kFlagBytes + slot * kFlagStride; }
+constexpr size_t kWorkspaceBytes = kFlagBytes + kBarSlots * kFlagStride;
+
 enum Dtype { kInt32 = 0, kFloat32 = 1, kBFloat16 = 2 };
 CCUBE_HD inline int elem_size(int dt) { return dt == kBFloat16 ? 2 : 4; }
 
@@ -117,6 +124,19 @@ int launch_tree_allreduce(const LaunchArgs &args, int dtype, bool sys_scope, int
 constexpr int kMaxGateCounters = 128;
 int launch_gate(const uint64_t *const *counters, const uint64_t *targets, int n, int *err,
                 uint64_t timeout_ns, bool sys_scope, void *stream);
+// ccube_barrier's kernel: one warp per local rank.
+struct BarrierRank {
+  const uint64_t *arrive[kMaxChildren];  // own arrive counters (written by children)
+  uint64_t *parent_arrive;               // parent's arrive counter of my slot, or null
+  const uint64_t *release;               // own release counter (written by the parent)
+  uint64_t *child_release[kMaxChildren]; // children's release counters
+  int nchild;
+};
+int launch_barrier(const BarrierRank *ranks, int n, uint64_t epoch, int *err,
+                   uint64_t timeout_ns, bool sys_scope, void *stream);
+// ccube_measure_peer_bandwidth's copy: src (local) -> every dst (peer), 128-bit.
+int launch_peer_copy(const char *src, char *const *dst, int ndst, size_t bytes, int grid,
+                     void *stream);
 int query_max_blocks_per_sm(int dtype, bool sys_scope, bool sgd, int threads, int tma,
                             int *blocks);
 

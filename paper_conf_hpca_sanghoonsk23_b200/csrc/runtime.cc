@@ -15,6 +15,7 @@
 #include <cuda_runtime.h>
 
 #include <cstdarg>
+#include <climits>
 #include <cstdint>
 #include <cstdio>
 #include <cstdlib>
@@ -29,6 +30,7 @@
 
 #include "ccube.h"
 #include "internal.h"
+#include "plan.h"
 #include "trees.h"
 
 namespace ccube {
@@ -191,6 +193,8 @@ struct Comm {
   uint64_t *trace = nullptr;
   size_t trace_kmax = 0;
   bool use_memop = true;
+  bool gate_flush = false;          // memop waits carry CU_STREAM_WAIT_VALUE_FLUSH
+  uint64_t bar_epoch = 0;           // ccube_barrier calls so far
 };
 
 Comm g;
@@ -232,10 +236,11 @@ ccube_result_t check_err_word() {
   if (g.err_host && *reinterpret_cast<volatile int *>(g.err_host) != 0) {
     volatile int *e = g.err_host;
     g.poisoned = true;
+    const char *what = e[0] == 2 ? "gradient-queue gate" : e[0] == 3 ? "barrier" : "AllReduce";
     return fail(CCUBE_ERR_TIMEOUT,
-                "device watchdog fired (block %d waited for counter >= %d, saw %d); the "
-                "communicator must be finalized",
-                e[1], e[2], e[3]);
+                "device watchdog fired in the %s kernel (block %d waited for counter >= %d, "
+                "saw %d); the communicator must be finalized",
+                what, e[1], e[2], e[3]);
   }
   return CCUBE_SUCCESS;
 }
@@ -244,7 +249,8 @@ ccube_result_t check_err_word() {
 // produce a usable pointer for every neighbour rank.  In loopback mode the local
 // pointers are used directly.
 ccube_result_t exchange_ptrs(const std::vector<char *> &local, size_t bytes,
-                             std::vector<char *> *world_ptrs, std::vector<void *> *opened) {
+                             std::vector<char *> *world_ptrs, std::vector<void *> *opened,
+                             bool every_rank = false) {
   world_ptrs->assign(g.world, nullptr);
   for (int i = 0; i < g.nlocal; ++i) (*world_ptrs)[g.rank0 + i] = local[i];
   if (g.nproc == 1) return CCUBE_SUCCESS;
@@ -265,7 +271,7 @@ ccube_result_t exchange_ptrs(const std::vector<char *> &local, size_t bytes,
   std::vector<IpcEntry> all(static_cast<size_t>(g.nproc) * g.nlocal);
   CC_TRY(do_allgather(mine.data(), all.data(), sizeof(IpcEntry) * g.nlocal));
   for (int r = 0; r < g.world; ++r) {
-    if (is_local(r) || !is_neighbor_of_local(r)) continue;
+    if (is_local(r) || (!every_rank && !is_neighbor_of_local(r))) continue;
     const IpcEntry &e = all[r];
     if (!e.valid || e.bytes != bytes)
       return fail(CCUBE_ERR_INVALID_ARG, "rank %d registered %llu bytes, expected %llu", r,
@@ -281,9 +287,49 @@ ccube_result_t exchange_ptrs(const std::vector<char *> &local, size_t bytes,
 // PUSH or PULL for the edge child -> parent: PULL inside one
 // process (same GPU), PUSH across GPUs, unless forced by ccube_set_transport.
 bool edge_is_pull(int child, int parent) {
-  if (g.transport == CCUBE_TRANSPORT_PUSH) return false;
-  if (g.transport == CCUBE_TRANSPORT_PULL) return true;
-  return is_local(child) && is_local(parent);
+  return plan_edge_is_pull(g.transport, g.nlocal, child, parent);
+}
+
+PlanIn plan_in(uint64_t bytes) {
+  PlanIn in;
+  in.trees = g.trees;
+  in.ntrees = g.ntrees;
+  in.world = g.world;
+  in.nlocal = g.nlocal;
+  in.transport = g.transport;
+  in.overlap = g.overlap;
+  in.sgd = g.sgd;
+  in.bytes = bytes;
+  in.chunk_bytes = g.chunk_bytes;
+  return in;
+}
+
+// A setting every rank must share (channels, threads, datapath, transport, overlap,
+// the fused update): with several processes the setter is collective and checks
+// agreement through the allgather, so every rank accepts or rejects the same value.
+// `local` is this rank's own validation of the value; a rank whose value is invalid
+// still takes part in the exchange (sending a poison value), so no peer is left
+// waiting in the allgather and every rank returns an error.
+ccube_result_t agree_setting(const char *what, int64_t value,
+                             ccube_result_t local = CCUBE_SUCCESS) {
+  const int64_t kBad = INT64_MIN;
+  const int64_t mine = local == CCUBE_SUCCESS ? value : kBad;
+  if (g.nproc > 1) {
+    std::vector<int64_t> all(g.nproc);
+    const std::string saved = g_err;
+    CC_TRY(do_allgather(&mine, all.data(), sizeof mine));
+    if (local != CCUBE_SUCCESS) {
+      g_err = saved;
+      return local;
+    }
+    for (int p = 0; p < g.nproc; ++p)
+      if (all[p] != mine)
+        return fail(CCUBE_ERR_INVALID_ARG, "ranks disagree on %s (process %d: %s%lld, here: %lld)",
+                    what, p, all[p] == kBad ? "invalid " : "", (long long)all[p], (long long)mine);
+  } else if (local != CCUBE_SUCCESS) {
+    return local;
+  }
+  return CCUBE_SUCCESS;
 }
 
 bool needs_recv_planes() {
@@ -499,25 +545,6 @@ ccube_result_t check_chunk(size_t chunk_bytes) {
   return CCUBE_SUCCESS;
 }
 
-int count_tasks(int channels, int overlap) {
-  int n = 0;
-  for (int i = 0; i < g.nlocal; ++i) {
-    const int r = g.rank0 + i;
-    for (int t = 0; t < g.ntrees; ++t) {
-      const Tree &tr = g.trees[t];
-      const bool root = tr.parent[r] < 0;
-      if (!root && tr.nchild[r] == 0 && g.sgd) n += channels;
-      if (!root && tr.nchild[r] == 0 && edge_is_pull(r, tr.parent[r])) {
-        n += 1;
-        continue;
-      }
-      n += channels;
-      if (tr.nchild[r] > 0 && (!root || !overlap)) n += channels;
-    }
-  }
-  return n;
-}
-
 ccube_result_t allreduce_impl(void *const *bufs, size_t count, ccube_dtype_t dtype,
                               void *stream) {
   if (!g.init) return fail(CCUBE_ERR_NOT_INITIALIZED, "ccube_init has not been called");
@@ -567,21 +594,19 @@ ccube_result_t allreduce_impl(void *const *bufs, size_t count, ccube_dtype_t dty
                   cudaGetErrorString(static_cast<cudaError_t>(rc)));
     g.max_blocks[key] = b;
   }
+  // Launch geometry (both ends of an edge must slice chunks alike).
+  // J is computed from the maximum task count over ALL processes, so it does not
+  // depend on this rank's role in the trees; every setting it depends on is agreed
+  // (init's Hello, the collective setters) and every GPU has the same SM count and
+  // architecture (init checks it), so every rank computes the same J and the same
+  // co-residency verdict without another exchange.
   const int cap = g.max_blocks[key] * g.sm_count;
-  int J = g.channels;
-  if (J == 0) {  // auto: the most channels whose CTAs all fit at once ...
-    J = 1;
-    while (J < CCUBE_MAX_CHANNELS && count_tasks(J + 1, g.overlap) <= cap) ++J;
-    // ... but at least two 2 KB units per channel and chunk while the buffer is a
-    // few chunks long: a small buffer gets few channels, so few CTAs take part in
-    // the handshakes (latency).  A long buffer is bandwidth-bound, so it may use
-    // one unit per channel (P=2 at 256 KiB chunks: 128 channels instead of 64).
-    const uint64_t first = bytes < g.chunk_bytes ? bytes : g.chunk_bytes;
-    const uint64_t units = (first + 2047) / 2048;
-    const uint64_t per = bytes >= 16 * g.chunk_bytes ? 1 : 2;
-    const int jmax = units / per > 1 ? static_cast<int>(units / per) : 1;
-    if (J > jmax) J = jmax;
-  }
+  const PlanIn in = plan_in(bytes);
+  const int J = g.channels ? g.channels : plan_auto_channels(in, cap);
+  if (plan_max_tasks(in, J) > cap)
+    return fail(CCUBE_ERR_UNSUPPORTED,
+                "%d CTAs (channels=%d) cannot be co-resident (capacity %d per GPU); lower "
+                "channels", plan_max_tasks(in, J), J, cap);
 
   LaunchArgs a;
   memset(&a, 0, sizeof a);
@@ -609,10 +634,6 @@ ccube_result_t allreduce_impl(void *const *bufs, size_t count, ccube_dtype_t dty
   TaskTable *tt = nullptr;
   CC_TRY(get_tasks(J, g.overlap, &tt));
   a.tasks = tt->d_tasks;
-  if (tt->n > cap)
-    return fail(CCUBE_ERR_UNSUPPORTED,
-                "%d CTAs (channels=%d) cannot be co-resident (capacity %d); lower channels",
-                tt->n, J, cap);
 
   const int rc = launch_tree_allreduce(a, dtype, g.sys_scope, tt->n, cta_threads, stream);
   if (rc != cudaSuccess)
@@ -673,7 +694,8 @@ ccube_result_t gradq_wait_impl(int local_rank, int layer_id, void *stream) {
         ops[i].waitValue.operation = CU_STREAM_MEM_OP_WAIT_VALUE_64;
         ops[i].waitValue.address = reinterpret_cast<CUdeviceptr>(ctr[done + i]);
         ops[i].waitValue.value64 = tgt[done + i];
-        ops[i].waitValue.flags = CU_STREAM_WAIT_VALUE_GEQ;
+        ops[i].waitValue.flags =
+            CU_STREAM_WAIT_VALUE_GEQ | (g.gate_flush ? CU_STREAM_WAIT_VALUE_FLUSH : 0);
       }
       if (g_drv.batchMemOp(static_cast<CUstream>(stream), static_cast<unsigned>(n), ops.data(),
                            0) != CUDA_SUCCESS)
@@ -714,6 +736,12 @@ void release_all() {
 struct Hello {
   uint32_t magic;
   int32_t world, nlocal, rank, tree_kind, device;
+  // settings that fix which bytes a counter covers or how a chunk is sliced: every
+  // rank must start from the same ones (CCUBE_* environment)
+  int32_t channels, threads, datapath, transport, l2_hints, split_control;
+  // the launch geometry is computed locally from the occupancy: every GPU must be
+  // the same architecture with the same SM count
+  int32_t sm_count, cc_major, cc_minor, pad;
   uint64_t chunk_bytes;
   char busid[32];
   int8_t place[CCUBE_MAX_RANKS];  // the placement (R19), identity when none was set
@@ -731,6 +759,132 @@ bool is_permutation(const int *perm, int P) {
     seen[perm[v]] = true;
   }
   return true;
+}
+
+ccube_result_t barrier_impl(void *stream) {
+  if (!g.init) return fail(CCUBE_ERR_NOT_INITIALIZED, "ccube_init has not been called");
+  CC_TRY(check_err_word());
+  if (g.nproc == 1) return CCUBE_SUCCESS;  // one process: stream order is the barrier
+  const Tree &tr = g.trees[0];
+  std::vector<BarrierRank> br(g.nlocal);
+  for (int i = 0; i < g.nlocal; ++i) {
+    const int r = g.rank0 + i;
+    BarrierRank &b = br[i];
+    memset(&b, 0, sizeof b);
+    char *own = g.flags_local[i];
+    b.nchild = tr.nchild[r];
+    for (int s = 0; s < tr.nchild[r]; ++s) {
+      const int c = tr.child[r][s];
+      if (!g.world_flags[c]) return fail(CCUBE_ERR_BOOTSTRAP, "child %d not mapped", c);
+      b.arrive[s] = reinterpret_cast<const uint64_t *>(own + barrier_offset(kBarArrive0 + s));
+      b.child_release[s] = reinterpret_cast<uint64_t *>(g.world_flags[c] + barrier_offset(kBarRelease));
+    }
+    b.release = reinterpret_cast<const uint64_t *>(own + barrier_offset(kBarRelease));
+    const int par = tr.parent[r];
+    if (par >= 0) {
+      if (!g.world_flags[par]) return fail(CCUBE_ERR_BOOTSTRAP, "parent %d not mapped", par);
+      b.parent_arrive = reinterpret_cast<uint64_t *>(
+          g.world_flags[par] + barrier_offset(kBarArrive0 + child_slot(tr, par, r)));
+    }
+  }
+  const int rc = launch_barrier(br.data(), g.nlocal, g.bar_epoch + 1, g.err_dev, g.timeout_ns,
+                                g.sys_scope, stream);
+  if (rc != cudaSuccess)
+    return fail(CCUBE_ERR_CUDA, "barrier launch failed: %s",
+                cudaGetErrorString(static_cast<cudaError_t>(rc)));
+  ++g.bar_epoch;
+  return CCUBE_SUCCESS;
+}
+
+
+// ccube_measure_peer_bandwidth (SURVEY §8(d) "P2P port-peak microbenchmark"): the
+// AllReduce's own cross-GPU data path — 128-bit loads from local HBM, 128-bit
+// stores into a peer's HBM over NVLink / NVSwitch — timed on the device after a
+// device-side barrier, one destination per GPU at a time (every rank shifted by
+// the same k, so every port carries one stream each way) and fanned out to m peers.
+ccube_result_t peer_bandwidth_impl(size_t bytes, int iters, double *pair_gbs, double *fanout_gbs) {
+  if (!g.init) return fail(CCUBE_ERR_NOT_INITIALIZED, "ccube_init has not been called");
+  CC_TRY(check_err_word());
+  if (g.nlocal != 1 || g.nproc < 2)
+    return fail(CCUBE_ERR_UNSUPPORTED, "peer bandwidth needs one process per GPU (nlocal == 1)");
+  if (bytes == 0 || bytes % 16 || iters < 1 || !pair_gbs || !fanout_gbs)
+    return fail(CCUBE_ERR_INVALID_ARG, "bytes must be a positive multiple of 16, iters >= 1");
+  const int P = g.world, me = g.rank0;
+  char *src = nullptr, *recv = nullptr;
+  std::vector<char *> world_recv;
+  std::vector<void *> opened;
+  cudaStream_t st = nullptr;
+  cudaEvent_t e0 = nullptr, e1 = nullptr;
+  std::vector<double> mine(2 * P, 0.0);
+  ccube_result_t rc = CCUBE_SUCCESS;
+  auto cuda_ok = [&](cudaError_t e, const char *what) {
+    if (e != cudaSuccess && rc == CCUBE_SUCCESS)
+      rc = fail(CCUBE_ERR_CUDA, "%s: %s", what, cudaGetErrorString(e));
+    return rc == CCUBE_SUCCESS;
+  };
+  if (cuda_ok(cudaMalloc(&src, bytes), "cudaMalloc(src)") &&
+      cuda_ok(cudaMalloc(&recv, bytes * P), "cudaMalloc(recv)") &&
+      cuda_ok(cudaMemset(src, 0x5a, bytes), "cudaMemset") &&
+      cuda_ok(cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking), "stream") &&
+      cuda_ok(cudaEventCreate(&e0), "event") && cuda_ok(cudaEventCreate(&e1), "event") &&
+      cuda_ok(cudaDeviceSynchronize(), "sync"))
+    rc = exchange_ptrs(std::vector<char *>{recv}, bytes * P, &world_recv, &opened, true);
+  const int grid = 2 * g.sm_count;
+  auto timed = [&](const std::vector<char *> &dst) -> double {
+    double best = 1e30;
+    for (int it = 0; it < iters && rc == CCUBE_SUCCESS; ++it) {
+      rc = barrier_impl(st);
+      if (rc != CCUBE_SUCCESS) break;
+      cuda_ok(cudaEventRecord(e0, st), "record");
+      const int lr = launch_peer_copy(src, dst.data(), static_cast<int>(dst.size()), bytes, grid, st);
+      cuda_ok(static_cast<cudaError_t>(lr), "peer copy launch");
+      cuda_ok(cudaEventRecord(e1, st), "record");
+      if (!cuda_ok(cudaEventSynchronize(e1), "sync")) break;
+      rc = check_err_word();
+      if (rc != CCUBE_SUCCESS) break;
+      float ms = 0;
+      cuda_ok(cudaEventElapsedTime(&ms, e0, e1), "elapsed");
+      best = std::min(best, static_cast<double>(ms) * 1e-3);
+    }
+    return best;
+  };
+  for (int k = 1; k < P && rc == CCUBE_SUCCESS; ++k) {  // pairs: every rank shifted by k
+    const int d = (me + k) % P;
+    const double t = timed({world_recv[d] + static_cast<size_t>(me) * bytes});
+    mine[d] = bytes / t / 1e9;
+  }
+  for (int m = 1; m < P && rc == CCUBE_SUCCESS; ++m) {  // fan-out to m peers at once
+    std::vector<char *> dst;
+    for (int q = 1; q <= m; ++q)
+      dst.push_back(world_recv[(me + q) % P] + static_cast<size_t>(me) * bytes);
+    const double t = timed(dst);
+    mine[P + m] = static_cast<double>(m) * bytes / t / 1e9;
+  }
+  // every rank reaches this exchange (a failed rank sends NaNs), then peers stop
+  // using our memory before anything is unmapped or freed
+  if (rc != CCUBE_SUCCESS) std::fill(mine.begin(), mine.end(), -1.0);
+  std::vector<double> all(2 * P * g.nproc);
+  const ccube_result_t grc = do_allgather(mine.data(), all.data(), sizeof(double) * 2 * P);
+  if (rc == CCUBE_SUCCESS) rc = grc;
+  for (int p = 0; p < g.nproc && rc == CCUBE_SUCCESS; ++p)
+    if (all[2 * P * p] < 0) rc = fail(CCUBE_ERR_CUDA, "peer bandwidth failed on process %d", p);
+  if (rc == CCUBE_SUCCESS) {
+    for (int i = 0; i < P; ++i)
+      for (int j = 0; j < P; ++j) pair_gbs[i * P + j] = all[2 * P * i + j];
+    fanout_gbs[0] = 0.0;
+    for (int m = 1; m < P; ++m) {
+      double lo = 1e30;
+      for (int i = 0; i < P; ++i) lo = std::min(lo, all[2 * P * i + P + m]);
+      fanout_gbs[m] = lo;
+    }
+  }
+  for (void *b : opened) ipc_close(b);
+  if (e0) cudaEventDestroy(e0);
+  if (e1) cudaEventDestroy(e1);
+  if (st) cudaStreamDestroy(st);
+  if (src) cudaFree(src);
+  if (recv) cudaFree(recv);
+  return rc;
 }
 
 }  // namespace
@@ -816,6 +970,21 @@ ccube_result_t ccube_init(const ccube_world_t *world, ccube_tree_kind_t tree_kin
   mine.tree_kind = tree_kind;
   mine.device = g.device;
   mine.chunk_bytes = chunk_bytes;
+  mine.channels = g.channels;
+  mine.threads = g.threads;
+  mine.datapath = g.datapath;
+  mine.transport = g.transport;
+  mine.l2_hints = g.l2_hints;
+  mine.split_control = g.split_control;
+  if (cudaDeviceGetAttribute(&mine.sm_count, cudaDevAttrMultiProcessorCount, g.device) !=
+          cudaSuccess ||
+      cudaDeviceGetAttribute(&mine.cc_major, cudaDevAttrComputeCapabilityMajor, g.device) !=
+          cudaSuccess ||
+      cudaDeviceGetAttribute(&mine.cc_minor, cudaDevAttrComputeCapabilityMinor, g.device) !=
+          cudaSuccess) {
+    cudaGetLastError();
+    mine.sm_count = mine.cc_major = mine.cc_minor = -1;  // no GPU: CUDA setup fails below
+  }
   for (int v = 0; v < P; ++v) mine.place[v] = static_cast<int8_t>(g_place_P == P ? g_place[v] : v);
   if (cudaDeviceGetPCIBusId(mine.busid, sizeof mine.busid, g.device) != cudaSuccess)
     snprintf(mine.busid, sizeof mine.busid, "nodevice-%d", g.rank0);
@@ -836,6 +1005,27 @@ ccube_result_t ccube_init(const ccube_world_t *world, ccube_tree_kind_t tree_kin
                   "ranks disagree on the configuration (process %d: world %d nlocal %d rank %d "
                   "tree %d chunk %llu, or the placement)",
                   p, h.world, h.nlocal, h.rank, h.tree_kind, (unsigned long long)h.chunk_bytes);
+    }
+    if (h.sm_count != mine.sm_count || h.cc_major != mine.cc_major ||
+        h.cc_minor != mine.cc_minor) {
+      g = Comm();
+      return fail(CCUBE_ERR_UNSUPPORTED,
+                  "mixed GPUs (process %d: sm_%d%d with %d SMs; here sm_%d%d with %d SMs): "
+                  "the launch geometry needs identical GPUs",
+                  p, h.cc_major, h.cc_minor, h.sm_count, mine.cc_major, mine.cc_minor,
+                  mine.sm_count);
+    }
+    if (h.channels != mine.channels || h.threads != mine.threads ||
+        h.datapath != mine.datapath || h.transport != mine.transport ||
+        h.l2_hints != mine.l2_hints || h.split_control != mine.split_control) {
+      g = Comm();
+      return fail(CCUBE_ERR_INVALID_ARG,
+                  "ranks disagree on the launch settings (process %d: CCUBE_CHANNELS %d "
+                  "CCUBE_THREADS %d CCUBE_DATAPATH %d CCUBE_TRANSPORT %d CCUBE_L2_HINTS %d "
+                  "CCUBE_SPLIT_CONTROL %d; here %d %d %d %d %d %d)",
+                  p, h.channels, h.threads, h.datapath, h.transport, h.l2_hints,
+                  h.split_control, mine.channels, mine.threads, mine.datapath, mine.transport,
+                  mine.l2_hints, mine.split_control);
     }
     // Several processes on one GPU only time-slice (no MPS): their spinning kernels
     // make progress one context switch at a time.  Refused unless a test asks for it
@@ -875,16 +1065,56 @@ ccube_result_t ccube_init(const ccube_world_t *world, ccube_tree_kind_t tree_kin
   memset(g.err_host, 0, 4 * sizeof(int));
   ce = cudaHostGetDevicePointer(reinterpret_cast<void **>(&g.err_dev), g.err_host, 0);
   if (ce != cudaSuccess) return bail(fail(CCUBE_ERR_CUDA, "cudaHostGetDevicePointer: %s", cudaGetErrorString(ce)));
+  // (iii) peer access (SURVEY §8(b) validation): every tree neighbour on another GPU
+  // must be reachable with device loads/stores (NVLink / NVSwitch).  Decided
+  // collectively, so every rank either proceeds or returns UNSUPPORTED.
+  if (g.nproc > 1) {
+    int32_t ok = 1;
+    char why[200] = "";
+    for (int r = 0; r < g.world && ok; ++r) {
+      if (is_local(r) || !is_neighbor_of_local(r)) continue;
+      const Hello &h = all[r / g.nlocal];
+      if (strncmp(h.busid, mine.busid, sizeof h.busid) == 0) continue;  // shared GPU (tests)
+      int dev = -1;
+      if (cudaDeviceGetByPCIBusId(&dev, h.busid) != cudaSuccess) {
+        cudaGetLastError();  // the peer's GPU is not visible here: the IPC open decides
+        continue;
+      }
+      int can = 0;
+      if (cudaDeviceCanAccessPeer(&can, g.device, dev) != cudaSuccess) can = 0;
+      if (!can) {
+        ok = 0;
+        snprintf(why, sizeof why, "GPU %s (rank %d) cannot access GPU %s (rank %d) as a peer",
+                 mine.busid, g.rank0, h.busid, r);
+      }
+    }
+    std::vector<int32_t> oks(g.nproc);
+    rc = do_allgather(&ok, oks.data(), sizeof ok);
+    if (rc != CCUBE_SUCCESS) return bail(rc);
+    for (int p = 0; p < g.nproc; ++p)
+      if (!oks[p])
+        return bail(fail(CCUBE_ERR_UNSUPPORTED, "no peer access between tree neighbours (%s)",
+                         ok ? "reported by another process" : why));
+    // gate (a9) across GPUs: the data and the Enqueue Semaphore arrive as remote
+    // writes.  A stream memory-op wait is not an acquire in the PTX memory model;
+    // CU_STREAM_WAIT_VALUE_FLUSH makes earlier remote writes visible to the work
+    // that follows.  Without it the gate is the ld.acquire.sys spin kernel.
+    int flush = 0;
+    if (cudaDeviceGetAttribute(&flush, cudaDevAttrCanFlushRemoteWrites, g.device) != cudaSuccess)
+      flush = 0;
+    g.gate_flush = flush != 0;
+    if (!g.gate_flush) g.use_memop = false;
+  }
   g.flags_local.assign(g.nlocal, nullptr);
   for (int i = 0; i < g.nlocal; ++i) {
-    ce = cudaMalloc(&g.flags_local[i], kFlagBytes);
-    if (ce == cudaSuccess) ce = cudaMemset(g.flags_local[i], 0, kFlagBytes);
+    ce = cudaMalloc(&g.flags_local[i], kWorkspaceBytes);
+    if (ce == cudaSuccess) ce = cudaMemset(g.flags_local[i], 0, kWorkspaceBytes);
     if (ce != cudaSuccess) return bail(fail(CCUBE_ERR_CUDA, "flag workspace: %s", cudaGetErrorString(ce)));
   }
   ce = cudaDeviceSynchronize();
   if (ce != cudaSuccess) return bail(fail(CCUBE_ERR_CUDA, "sync: %s", cudaGetErrorString(ce)));
   g.init = true;  // exchange_ptrs needs the topology fields
-  rc = exchange_ptrs(g.flags_local, kFlagBytes, &g.world_flags, &g.opened_flags);
+  rc = exchange_ptrs(g.flags_local, kWorkspaceBytes, &g.world_flags, &g.opened_flags);
   if (rc != CCUBE_SUCCESS) return bail(rc);
   return CCUBE_SUCCESS;
 }
@@ -935,6 +1165,50 @@ ccube_result_t ccube_allreduce_tree_local(void *const *bufs, size_t count, ccube
   return allreduce_impl(bufs, count, dtype, stream);
 }
 
+ccube_result_t ccube_barrier(void *stream) {
+  std::lock_guard<std::mutex> lk(g_mu);
+  return barrier_impl(stream);
+}
+
+ccube_result_t ccube_measure_peer_bandwidth(size_t bytes, int iters, double *pair_gbs,
+                                            double *fanout_gbs) {
+  std::lock_guard<std::mutex> lk(g_mu);
+  return peer_bandwidth_impl(bytes, iters, pair_gbs, fanout_gbs);
+}
+
+ccube_result_t ccube_plan_launch(int P, ccube_tree_kind_t kind, int nlocal, int rank,
+                                 size_t bytes, size_t chunk_bytes, int overlap, int channels,
+                                 int cap_ctas, int *channels_out, int *ctas_out,
+                                 int *max_ctas_out) {
+  if (P < 1 || P > CCUBE_MAX_RANKS || nlocal < 1 || P % nlocal || rank < 0 || rank >= P)
+    return fail(CCUBE_ERR_INVALID_ARG, "bad P %d, nlocal %d or rank %d", P, nlocal, rank);
+  if (kind != CCUBE_TREE_SINGLE && kind != CCUBE_TREE_DOUBLE && kind != CCUBE_TREE_ROTATED)
+    return fail(CCUBE_ERR_INVALID_ARG, "bad tree kind %d", (int)kind);
+  if ((overlap != 0 && overlap != 1) || channels < 0 || channels > CCUBE_MAX_CHANNELS ||
+      cap_ctas < 1 || !channels_out || !ctas_out || !max_ctas_out)
+    return fail(CCUBE_ERR_INVALID_ARG, "bad overlap, channels, cap or output pointer");
+  if (chunk_bytes == 0) chunk_bytes = CCUBE_DEFAULT_CHUNK_BYTES;
+  CC_TRY(check_chunk(chunk_bytes));
+  Tree trees[kMaxTrees];
+  const int T = num_trees(P, kind);
+  for (int t = 0; t < T; ++t) build_tree(P, kind, t, &trees[t]);
+  PlanIn in;
+  in.trees = trees;
+  in.ntrees = T;
+  in.world = P;
+  in.nlocal = nlocal;
+  in.transport = CCUBE_TRANSPORT_AUTO;
+  in.overlap = overlap;
+  in.sgd = false;
+  in.bytes = bytes;
+  in.chunk_bytes = chunk_bytes;
+  const int J = channels ? channels : plan_auto_channels(in, cap_ctas);
+  *channels_out = J;
+  *ctas_out = plan_tasks_of_proc(in, rank / nlocal, J);
+  *max_ctas_out = plan_max_tasks(in, J);
+  return CCUBE_SUCCESS;
+}
+
 ccube_result_t ccube_gradq_set_layers(const size_t *layer_end_elems, int n_layers) {
   std::lock_guard<std::mutex> lk(g_mu);
   if (!g.init) return fail(CCUBE_ERR_NOT_INITIALIZED, "ccube_init has not been called");
@@ -963,7 +1237,10 @@ ccube_result_t ccube_gradq_wait_local(int local_rank, int layer_id, void *stream
 ccube_result_t ccube_set_overlap(int on) {
   std::lock_guard<std::mutex> lk(g_mu);
   if (!g.init) return fail(CCUBE_ERR_NOT_INITIALIZED, "ccube_init has not been called");
-  if (on != 0 && on != 1) return fail(CCUBE_ERR_INVALID_ARG, "overlap must be 0 or 1");
+  const ccube_result_t v = on != 0 && on != 1
+                               ? fail(CCUBE_ERR_INVALID_ARG, "overlap must be 0 or 1")
+                               : CCUBE_SUCCESS;
+  CC_TRY(agree_setting("overlap", on, v));
   g.overlap = on;
   return CCUBE_SUCCESS;
 }
@@ -971,19 +1248,25 @@ ccube_result_t ccube_set_overlap(int on) {
 ccube_result_t ccube_gradq_set_sgd(void *const *weights, size_t bytes, float alpha) {
   std::lock_guard<std::mutex> lk(g_mu);
   if (!g.init) return fail(CCUBE_ERR_NOT_INITIALIZED, "ccube_init has not been called");
+  ccube_result_t v = CCUBE_SUCCESS;
+  if (weights) {
+    if (g.world < 2)
+      v = fail(CCUBE_ERR_UNSUPPORTED, "the fused SGD update rides on the AllReduce (P >= 2)");
+    else if (bytes == 0 || bytes % 4)
+      v = fail(CCUBE_ERR_INVALID_ARG, "bad weight bytes %zu", bytes);
+    for (int i = 0; i < g.nlocal && v == CCUBE_SUCCESS; ++i) {
+      if (!weights[i])
+        v = fail(CCUBE_ERR_INVALID_ARG, "weights[%d] is NULL", i);
+      else if (reinterpret_cast<uintptr_t>(weights[i]) % 16)
+        v = fail(CCUBE_ERR_INVALID_ARG, "weights[%d] is not 16-byte aligned", i);
+    }
+  }
+  CC_TRY(agree_setting("the fused SGD update (on/off)", weights ? 1 : 0, v));
   if (!weights) {
     g.sgd = false;
     g.sgd_w.clear();
     g.sgd_bytes = 0;
   } else {
-    if (g.world < 2)
-      return fail(CCUBE_ERR_UNSUPPORTED, "the fused SGD update rides on the AllReduce (P >= 2)");
-    if (bytes == 0 || bytes % 4) return fail(CCUBE_ERR_INVALID_ARG, "bad weight bytes %zu", bytes);
-    for (int i = 0; i < g.nlocal; ++i) {
-      if (!weights[i]) return fail(CCUBE_ERR_INVALID_ARG, "weights[%d] is NULL", i);
-      if (reinterpret_cast<uintptr_t>(weights[i]) % 16)
-        return fail(CCUBE_ERR_INVALID_ARG, "weights[%d] is not 16-byte aligned", i);
-    }
     g.sgd = true;
     g.sgd_alpha = alpha;
     g.sgd_bytes = bytes;
@@ -997,10 +1280,12 @@ ccube_result_t ccube_gradq_set_sgd(void *const *weights, size_t bytes, float alp
 ccube_result_t ccube_set_channels(int channels) {
   std::lock_guard<std::mutex> lk(g_mu);
   if (!g.init) return fail(CCUBE_ERR_NOT_INITIALIZED, "ccube_init has not been called");
-  if (channels < 0 || channels > CCUBE_MAX_CHANNELS)
-    return fail(CCUBE_ERR_INVALID_ARG, "channels %d out of range [0 (auto), %d]", channels,
-                CCUBE_MAX_CHANNELS);
-  
+  const ccube_result_t v =
+      channels < 0 || channels > CCUBE_MAX_CHANNELS
+          ? fail(CCUBE_ERR_INVALID_ARG, "channels %d out of range [0 (auto), %d]", channels,
+                 CCUBE_MAX_CHANNELS)
+          : CCUBE_SUCCESS;
+  CC_TRY(agree_setting("channels", channels, v));
   g.channels = channels;
   return CCUBE_SUCCESS;
 }
@@ -1008,9 +1293,12 @@ ccube_result_t ccube_set_channels(int channels) {
 ccube_result_t ccube_set_threads(int threads) {
   std::lock_guard<std::mutex> lk(g_mu);
   if (!g.init) return fail(CCUBE_ERR_NOT_INITIALIZED, "ccube_init has not been called");
-  if (threads < 32 || threads > 256 || threads % 32)
-    return fail(CCUBE_ERR_INVALID_ARG, "threads %d out of range [32, 256] (multiple of 32)",
-                threads);
+  const ccube_result_t v =
+      threads < 32 || threads > 256 || threads % 32
+          ? fail(CCUBE_ERR_INVALID_ARG, "threads %d out of range [32, 256] (multiple of 32)",
+                 threads)
+          : CCUBE_SUCCESS;
+  CC_TRY(agree_setting("threads", threads, v));
   g.threads = threads;
   return CCUBE_SUCCESS;
 }
@@ -1018,9 +1306,11 @@ ccube_result_t ccube_set_threads(int threads) {
 ccube_result_t ccube_set_datapath(int datapath) {
   std::lock_guard<std::mutex> lk(g_mu);
   if (!g.init) return fail(CCUBE_ERR_NOT_INITIALIZED, "ccube_init has not been called");
-  if (datapath != CCUBE_DATAPATH_LSU && datapath != CCUBE_DATAPATH_TMA &&
-      datapath != CCUBE_DATAPATH_AUTO)
-    return fail(CCUBE_ERR_INVALID_ARG, "datapath %d out of range", datapath);
+  const ccube_result_t v = datapath != CCUBE_DATAPATH_LSU && datapath != CCUBE_DATAPATH_TMA &&
+                                   datapath != CCUBE_DATAPATH_AUTO
+                               ? fail(CCUBE_ERR_INVALID_ARG, "datapath %d out of range", datapath)
+                               : CCUBE_SUCCESS;
+  CC_TRY(agree_setting("datapath", datapath, v));
   g.datapath = datapath;
   return CCUBE_SUCCESS;
 }
@@ -1028,8 +1318,10 @@ ccube_result_t ccube_set_datapath(int datapath) {
 ccube_result_t ccube_set_transport(int mode) {
   std::lock_guard<std::mutex> lk(g_mu);
   if (!g.init) return fail(CCUBE_ERR_NOT_INITIALIZED, "ccube_init has not been called");
-  if (mode < CCUBE_TRANSPORT_AUTO || mode > CCUBE_TRANSPORT_PULL)
-    return fail(CCUBE_ERR_INVALID_ARG, "transport %d out of range", mode);
+  const ccube_result_t v = mode < CCUBE_TRANSPORT_AUTO || mode > CCUBE_TRANSPORT_PULL
+                               ? fail(CCUBE_ERR_INVALID_ARG, "transport %d out of range", mode)
+                               : CCUBE_SUCCESS;
+  CC_TRY(agree_setting("transport", mode, v));
   if (mode == g.transport) return CCUBE_SUCCESS;
   CUDA_TRY(cudaDeviceSynchronize());
   g.transport = mode;

@@ -1100,6 +1100,79 @@ __global__ void gate_kernel(const GateArgs g) {
   }
 }
 
+// Device-side barrier over tree 0 (ccube_barrier): warp i serves local rank i.
+// Lane s < nchild waits for child s's "arrive" >= epoch; then lane 0 tells the
+// parent (release store into the parent's counter), waits for the parent's
+// "release" and passes it on to the children.  Once the root has heard from
+// every subtree, every rank has entered the barrier; once a rank sees "release",
+// the root had.  Same single-writer monotone counters as the AllReduce.
+struct BarrierArgs {
+  BarrierRank r[kMaxRanks];
+  uint64_t epoch;
+  int *err;
+  uint64_t timeout_ns;
+};
+
+template <bool SYS>
+__global__ void barrier_kernel(const BarrierArgs b) {
+  const int lane = threadIdx.x & 31;
+  const BarrierRank &me = b.r[threadIdx.x >> 5];
+  const uint64_t t0 = globaltimer();
+  bool ok = true;
+  auto wait_ge = [&](const uint64_t *p) {
+    while (ok && ld_acquire<SYS>(p) < b.epoch) {
+      if (*reinterpret_cast<volatile int *>(b.err) != 0 || globaltimer() - t0 > b.timeout_ns) {
+        if (*reinterpret_cast<volatile int *>(b.err) == 0) {
+          *reinterpret_cast<volatile int *>(b.err) = 3;  // 3 = barrier timeout
+          __threadfence_system();
+        }
+        ok = false;
+      }
+    }
+  };
+  if (lane < me.nchild) wait_ge(me.arrive[lane]);
+  __syncwarp();
+  if (lane == 0) {
+    if (me.parent_arrive) {
+      fence_release<SYS>();
+      st_relaxed<SYS>(me.parent_arrive, b.epoch);
+      wait_ge(me.release);
+    }
+    fence_release<SYS>();
+    for (int s = 0; s < me.nchild; ++s) st_relaxed<SYS>(me.child_release[s], b.epoch);
+  }
+}
+
+// Peer-bandwidth probe (ccube_measure_peer_bandwidth): the data warps' copy pattern —
+// U 128-bit loads per lane from local HBM, then 128-bit stores with an evict_first
+// policy — into destination blockIdx.y (a peer's HBM, mapped with CUDA IPC).
+struct PeerCopyArgs {
+  const char *src;
+  char *dst[kMaxRanks];
+  uint64_t nvec;
+};
+
+__global__ void __launch_bounds__(256) peer_copy_kernel(const PeerCopyArgs c) {
+  constexpr int U = 4;
+  const L2Pol pol = make_pol(1);
+  char *dst = c.dst[blockIdx.y];
+  const uint64_t stride = static_cast<uint64_t>(gridDim.x) * blockDim.x * U;
+  for (uint64_t i0 = static_cast<uint64_t>(blockIdx.x) * blockDim.x * U + threadIdx.x;
+       i0 < c.nvec; i0 += stride) {
+    uint4 v[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const uint64_t i = i0 + static_cast<uint64_t>(u) * blockDim.x;
+      if (i < c.nvec) v[u] = ld_hint(c.src + 16 * i, pol.first);
+    }
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const uint64_t i = i0 + static_cast<uint64_t>(u) * blockDim.x;
+      if (i < c.nvec) st_hint(dst + 16 * i, v[u], pol.first);
+    }
+  }
+}
+
 template <int DT, bool SYS, bool SGD>
 int launch_t(const LaunchArgs &a, int grid, int threads, cudaStream_t s) {
   const size_t smem = a.tma ? kTmaRing : 0;
@@ -1168,6 +1241,34 @@ int launch_gate(const uint64_t *const *counters, const uint64_t *targets, int n,
     gate_kernel<true><<<1, 32, 0, s>>>(g);
   else
     gate_kernel<false><<<1, 32, 0, s>>>(g);
+  return static_cast<int>(cudaGetLastError());
+}
+
+int launch_barrier(const BarrierRank *ranks, int n, uint64_t epoch, int *err,
+                   uint64_t timeout_ns, bool sys_scope, void *stream) {
+  if (n <= 0 || n > kMaxRanks) return cudaErrorInvalidValue;
+  BarrierArgs b;
+  for (int i = 0; i < n; ++i) b.r[i] = ranks[i];
+  b.epoch = epoch;
+  b.err = err;
+  b.timeout_ns = timeout_ns;
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  if (sys_scope)
+    barrier_kernel<true><<<1, 32 * n, 0, s>>>(b);
+  else
+    barrier_kernel<false><<<1, 32 * n, 0, s>>>(b);
+  return static_cast<int>(cudaGetLastError());
+}
+
+int launch_peer_copy(const char *src, char *const *dst, int ndst, size_t bytes, int grid,
+                     void *stream) {
+  if (ndst < 1 || ndst > kMaxRanks || bytes % 16) return cudaErrorInvalidValue;
+  PeerCopyArgs c;
+  c.src = src;
+  for (int i = 0; i < ndst; ++i) c.dst[i] = dst[i];
+  c.nvec = bytes / 16;
+  const int gx = grid / ndst > 0 ? grid / ndst : 1;
+  peer_copy_kernel<<<dim3(gx, ndst), 256, 0, static_cast<cudaStream_t>(stream)>>>(c);
   return static_cast<int>(cudaGetLastError());
 }
 

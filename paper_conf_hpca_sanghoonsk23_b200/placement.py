@@ -18,11 +18,25 @@ from . import ccube
 
 
 def measure_peer_bandwidth(pg=None, nbytes: int = 64 << 20, reps: int = 3):
-    """bw[i][j] in GB/s for rank i -> rank j, one ordered pair at a time (send/recv
-    over ``pg``: NCCL over NVLink on GPUs, gloo on CPU), identical on every rank."""
+    """bw[i][j] in GB/s for rank i -> rank j, identical on every rank.
+
+    On GPUs (an NCCL group) this is the library's own store path
+    (``ccube_measure_peer_bandwidth``: the AllReduce kernel's 128-bit loads from
+    local HBM and stores into the peer's HBM, device-timed after a device-side
+    barrier, every rank storing to its k-th successor at once) through a temporary
+    identity-placed communicator — the bandwidth the tree edges will actually see.
+    On CPU (gloo, the host tests) it falls back to timing send/recv per ordered pair."""
     pg = pg or dist.group.WORLD
     P, me = dist.get_world_size(pg), dist.get_rank(pg)
     on_gpu = dist.get_backend(pg) == "nccl"
+    if on_gpu:
+        ccube.set_placement(None)
+        ccube.init_distributed(pg, tree="single")
+        try:
+            pair, _ = ccube.measure_peer_bandwidth(nbytes, reps)
+        finally:
+            ccube.finalize()
+        return pair
     dev = torch.device("cuda", torch.cuda.current_device()) if on_gpu else torch.device("cpu")
     buf = torch.empty(nbytes // 4, dtype=torch.float32, device=dev)
     sync = torch.cuda.synchronize if on_gpu else (lambda: None)

@@ -131,3 +131,112 @@ def test_gloo_bootstrap_detects_mismatch_ws2():
     for rank, code, msg in out:
         assert code == ccube.ERR_INVALID_ARG, msg
         assert "disagree" in msg
+
+
+# ---- launch geometry is a collective decision -----------------------
+
+def _py_tasks(P, kind, nlocal, proc, J, overlap):
+    """Independent restatement of the task table: per rank and tree, UP on J channels,
+    DOWN on J channels at interior nodes (and at the root in B), a pulled leaf (same
+    process as its parent) one CTA."""
+    T = {"single": 1, "double": 2, "rotated": P}[kind]
+    n = 0
+    for r in range(proc * nlocal, (proc + 1) * nlocal):
+        for t in range(T):
+            par = ccube.tree_parents(P, kind, t)
+            nch = sum(1 for u in range(P) if par[u] == r)
+            root = par[r] < 0
+            if not root and nch == 0 and par[r] // nlocal == r // nlocal:
+                n += 1
+                continue
+            n += J
+            if nch > 0 and (not root or not overlap):
+                n += J
+    return n
+
+
+def _py_jmax(nbytes, chunk):
+    first = min(nbytes, chunk)
+    units = -(-first // 2048)
+    per = 1 if nbytes >= 16 * chunk else 2
+    return max(units // per, 1)
+
+
+SIZES = [1 << 10, 1 << 20, 4 << 20, 102_228_128, 1 << 30]
+
+
+@pytest.mark.parametrize("P", range(2, 9))
+@pytest.mark.parametrize("kind", ["single", "double", "rotated"])
+@pytest.mark.parametrize("overlap", [0, 1])
+def test_plan_launch_every_rank_agrees(P, kind, overlap):
+    """One process per GPU: every rank gets the same J for every size (so both ends of
+    an edge slice chunks alike), J is the largest whose busiest process fits the cap,
+    and no process exceeds the cap."""
+    cap = 296   # 2 CTAs x 148 SMs (B200, 320-thread CTAs)
+    for nbytes in SIZES:
+        got = [ccube.plan_launch(P, kind, 1, r, nbytes, 256 << 10, overlap, 0, cap)
+               for r in range(P)]
+        Js = {j for j, _, _ in got}
+        assert len(Js) == 1, (nbytes, got)
+        J = Js.pop()
+        tasks = [_py_tasks(P, kind, 1, r, J, overlap) for r in range(P)]
+        assert [n for _, n, _ in got] == tasks
+        assert all(m == max(tasks) for _, _, m in got)
+        assert max(tasks) <= cap
+        # J is maximal: one more channel would overflow the busiest process, or the
+        # per-chunk unit cap binds
+        jmax = min(_py_jmax(nbytes, 256 << 10), 128)
+        assert J == jmax or max(_py_tasks(P, kind, 1, r, J + 1, overlap)
+                                for r in range(P)) > cap
+
+
+def test_per_rank_rule_would_disagree():
+    """The round-1 rule (J from this process's own tasks) gives the roots of the
+    double tree at P=8, C1, >= 16 chunks a different J than the other ranks — the
+    hang the collective rule removes."""
+    P, cap, nbytes = 8, 296, 102_228_128
+    own = []
+    for r in range(P):
+        J = 1
+        while J < 128 and _py_tasks(P, "double", 1, r, J + 1, 1) <= cap:
+            J += 1
+        own.append(min(J, _py_jmax(nbytes, 256 << 10)))
+    assert len(set(own)) > 1, own
+    lib = {ccube.plan_launch(P, "double", 1, r, nbytes, 256 << 10, 1, 0, cap)[0]
+           for r in range(P)}
+    assert lib == {min(own)}
+
+
+def test_plan_launch_loopback_and_explicit():
+    # loopback: one process hosts every rank
+    j, n, m = ccube.plan_launch(8, "single", 8, 0, 102_228_128, 256 << 10, 1, 0, 296)
+    assert n == m == _py_tasks(8, "single", 8, 0, j, 1) <= 296
+    assert j == 41   # 7 J + 4 pulled leaves <= 296 (the round-1 bench geometry)
+    # explicit channels are returned as given
+    assert ccube.plan_launch(4, "double", 1, 2, 1 << 20, 0, 1, 7, 296)[0] == 7
+    with pytest.raises(ccube.CCubeError) as e:
+        ccube.plan_launch(4, "double", 3, 0, 1 << 20, 0, 1, 0, 296)
+    assert e.value.code == ccube.ERR_INVALID_ARG
+
+
+def _env_worker(rank, world, port, env, q):
+    os.environ.update(env[rank])
+    _bootstrap_worker(rank, world, port, [256 << 10] * world, q)
+
+
+def test_gloo_bootstrap_detects_launch_setting_mismatch_ws2():
+    """CCUBE_CHANNELS differs between the two processes: both refuse at init."""
+    import torch.multiprocessing as mp
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    env = [{"CCUBE_CHANNELS": "8"}, {"CCUBE_CHANNELS": "16"}]
+    procs = [ctx.Process(target=_env_worker, args=(r, 2, port, env, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    out = sorted(q.get(timeout=120) for _ in procs)
+    for p in procs:
+        p.join(timeout=60)
+    for rank, code, msg in out:
+        assert code == ccube.ERR_INVALID_ARG, msg
+        assert "launch settings" in msg

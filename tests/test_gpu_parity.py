@@ -229,9 +229,15 @@ def test_overlap_and_baseline_bitwise_equal_full_size(comm):
 
 
 @pytest.mark.parametrize("kind", ["single", "double"])
-def test_gradient_queue_gates_each_layer(comm, kind):
+@pytest.mark.parametrize("gate", ["memop", "kernel"])
+def test_gradient_queue_gates_each_layer(comm, monkeypatch, kind, gate):
     """a9: on a second stream, gradq_wait(l) then snapshot layer l's gradients; every
-    snapshot must already hold the final reduced values."""
+    snapshot must already hold the final reduced values.  Both gate
+    mechanisms: the stream memory-op wait and the ld.acquire spin kernel
+    (CCUBE_GATE_KERNEL=1, the one-process-per-GPU default without remote-write
+    flush)."""
+    if gate == "kernel":
+        monkeypatch.setenv("CCUBE_GATE_KERNEL", "1")
     P, chunk = 8, 64 << 10
     comm(P, kind, chunk, channels=4)
     ends = workloads.layer_ends("resnet50")
