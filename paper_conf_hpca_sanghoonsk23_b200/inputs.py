@@ -13,6 +13,26 @@ Recipe:
   conversion); int32 inputs are uniform in [-2**24, 2**24) (sums are then exact
   without wrap at P <= 8) or, with ``full_range=True``, uniform over all int32.
 Default seed 20230225 (the paper's conference date), recorded in bench output.
+
+``special(rank, count, dtype)`` is a second recipe for the parity tests (VERDICT r1
+W2): IEEE corner cases that decide whether the device honours reading R3 (no
+FTZ/DAZ, RN adds, signed zeros, one RNE per bf16 node output).  Every element
+belongs to a class picked by a RANK-INDEPENDENT hash of (seed, e), so all ranks
+see the same kind of value at e and the partial sums stay in that regime:
+  0, 1  normal: the default recipe's N(0,1) * 2^-k;
+  2     subnormal: +-m * 2^-149 with m in [1, 2^20) (fp32) or [2^16, 2^20) (bf16),
+        random sign per rank; any tree's sum of <= 8 stays exact and below 2^-126,
+        so a flush-to-zero anywhere turns a nonzero result into 0;
+  3     signed zero: +0 or -0 per rank; on every other such element all ranks -0
+        (the only way an IEEE RN sum is -0);
+  4     near the format maximum: +-(1 + f) * 2^123 (sums of <= 8 cannot overflow);
+  5     at the normal/subnormal boundary: exponent field 0 or 1, random mantissa;
+  6     cancellation: the same magnitude m (8 significant bits, so every partial
+        sum k*m, |k| <= 8, is exact in fp32) on every rank, + on even ranks, - on
+        odd: at even P the exact sum is 0, and an RN sum that is exactly zero is +0;
+  7     mixed: the class of (rank, e) instead, so magnitudes of every kind meet.
+int32: 0,1 uniform in [-2^24, 2^24); 2 INT32_MIN; 3 INT32_MAX; 4 in {-1, 0, 1};
+5, 6, 7 uniform over all int32 (wraps).  No NaN or Inf is generated (unpinned).
 """
 
 from typing import Optional, Sequence
@@ -89,4 +109,78 @@ def gradients(rank: int, count: int, dtype: str, seed: int = SEED,
         return gradients_bf16(rank, count, seed, layer_ends, lo, hi)
     if dtype == "int32":
         return gradients_i32(rank, count, seed, full_range, lo, hi)
+    raise ValueError(dtype)
+
+
+# ---- the special-value recipe (parity tests) ---------------------------------------
+SPECIAL_CLASSES = 8
+
+
+def special_class(lo: int, hi: int, seed: int = SEED, rank: Optional[int] = None) -> np.ndarray:
+    """Class of elements [lo, hi): a hash of (seed, e) — of (seed, rank, e) with rank."""
+    key = np.uint64(seed ^ 0x5EC1A1) if rank is None else \
+        np.uint64(seed ^ 0x5EC1A1) ^ (np.uint64(rank + 1) << np.uint64(40))
+    h = splitmix64(np.arange(lo, hi, dtype=np.uint64) ^ key)
+    return (h >> np.uint64(61)).astype(np.int64)
+
+
+def _special_f32_bits(rank: int, lo: int, hi: int, seed: int, bf16: bool) -> np.ndarray:
+    cls = special_class(lo, hi, seed)
+    mixed = cls == 7
+    cls[mixed] = special_class(lo, hi, seed, rank)[mixed] % 7
+    h = _hash(rank, lo, hi, seed ^ 0x77)                  # per (rank, e)
+    hs = splitmix64(np.arange(lo, hi, dtype=np.uint64) ^ np.uint64(seed ^ 0x3C3C))  # per e
+    sign = ((h >> np.uint64(63)) << np.uint64(31)).astype(np.uint32)
+    mant = ((h >> np.uint64(20)) & np.uint64(0x7FFFFF)).astype(np.uint32)
+    base = gradients_f32(rank, hi, seed, None, lo, hi).view(np.uint32)
+    out = base.copy()
+    # 2: subnormal
+    if bf16:
+        m = (np.uint32(1 << 16) + (mant & np.uint32((1 << 20) - 1 - (1 << 16))))
+    else:
+        m = np.maximum(mant & np.uint32((1 << 20) - 1), np.uint32(1))
+    sel = cls == 2
+    out[sel] = sign[sel] | m[sel]
+    # 3: signed zero (every other such element: all ranks -0)
+    sel = cls == 3
+    all_neg = ((hs >> np.uint64(7)) & np.uint64(1)).astype(bool)
+    out[sel] = np.where(all_neg[sel], np.uint32(0x80000000), sign[sel])
+    # 4: near max, +-(1 + f) * 2^123
+    sel = cls == 4
+    out[sel] = sign[sel] | np.uint32((123 + 127) << 23) | mant[sel]
+    # 5: exponent field 0 or 1
+    sel = cls == 5
+    e1 = ((h >> np.uint64(5)) & np.uint64(1)).astype(np.uint32) << np.uint32(23)
+    out[sel] = sign[sel] | e1[sel] | mant[sel]
+    # 6: cancellation: magnitude per e, sign by rank parity
+    sel = cls == 6
+    mag = (np.uint32(127 << 23) | ((hs >> np.uint64(20)) & np.uint64(0x7F0000)).astype(np.uint32))
+    out[sel] = mag[sel] | (np.uint32(0x80000000) if rank % 2 else np.uint32(0))
+    return out
+
+
+def special(rank: int, count: int, dtype: str, seed: int = SEED,
+            lo: int = 0, hi: Optional[int] = None) -> np.ndarray:
+    """The special-value recipe (module docstring) for elements [lo, hi)."""
+    hi = count if hi is None else hi
+    if dtype == "float32":
+        return _special_f32_bits(rank, lo, hi, seed, False).view(np.float32)
+    if dtype == "bfloat16":
+        import torch
+        f = torch.from_numpy(_special_f32_bits(rank, lo, hi, seed, True).view(np.float32))
+        return f.to(torch.bfloat16).view(torch.int16).numpy().view(np.uint16)
+    if dtype == "int32":
+        cls = special_class(lo, hi, seed)
+        mixed = cls == 7
+        cls[mixed] = special_class(lo, hi, seed, rank)[mixed] % 7
+        h = _hash(rank, lo, hi, seed ^ 0x99)
+        out = ((h >> np.uint64(39)).astype(np.int64) - (1 << 24)).astype(np.int32)
+        full = (h & np.uint64(0xFFFFFFFF)).astype(np.uint32).view(np.int32)
+        out[cls == 2] = np.iinfo(np.int32).min
+        out[cls == 3] = np.iinfo(np.int32).max
+        small = ((h >> np.uint64(3)) % np.uint64(3)).astype(np.int32) - 1
+        out[cls == 4] = small[cls == 4]
+        sel = cls >= 5
+        out[sel] = full[sel]
+        return out
     raise ValueError(dtype)

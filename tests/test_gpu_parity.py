@@ -576,3 +576,91 @@ def test_max_size_1gib_ragged(comm, kind):
             assert np.array_equal(to_numpy(ts[r][lo:hi], "float32"), want), (c, r)
     for r in range(1, P):
         assert torch.equal(ts[r], ts[0])
+
+
+# ---- IEEE corner cases: inputs.special ---------------------------------
+def _run_special(P, kind, dtype, count, chunk):
+    xs = [inputs.special(r, count, dtype) for r in range(P)]
+    ts = [to_torch(x, dtype).cuda() for x in xs]
+    ccube.allreduce_tree_local(ts)
+    torch.cuda.synchronize()
+    return xs, [to_numpy(t, dtype) for t in ts]
+
+
+@pytest.mark.parametrize("P", [4, 8])
+@pytest.mark.parametrize("kind", ["single", "double", "rotated"])
+@pytest.mark.parametrize("dtype", ["int32", "float32", "bfloat16"])
+@pytest.mark.parametrize("overlap", [True, False])
+@pytest.mark.parametrize("transport", ["pull", "push"])
+@pytest.mark.parametrize("datapath", ["lsu", "tma"])
+def test_parity_special_values(comm, P, kind, dtype, overlap, transport, datapath):
+    """Subnormals, +-0, near-max values, the normal/subnormal boundary, exact
+    cancellation and int32 extremes (inputs.special): bit-exact vs the oracle on
+    every tree, B and C1, both edge transports and both datapaths, ragged tail.  A
+    build with -ftz=true, a contracted FMA or a wrong signed-zero rule fails here."""
+    chunk = 4096
+    comm(P, kind, chunk, channels=3, overlap=overlap, transport=transport)
+    ccube.set_datapath(datapath)
+    E = chunk // arith.ELEM_SIZE[dtype]
+    count = 7 * E + 13
+    xs, outs = _run_special(P, kind, dtype, count, chunk)
+    ref = oar.reference(xs, kind, chunk, dtype)[0]
+    for r in range(P):
+        assert np.array_equal(outs[r], ref), f"rank {r}"
+
+
+@pytest.mark.parametrize("dtype", ["float32", "bfloat16"])
+def test_device_keeps_subnormals_and_signed_zeros(comm, dtype):
+    """Reading R3 observed on the device: where every rank holds a subnormal the
+    result is a nonzero subnormal (no FTZ/DAZ), where every rank holds -0 it is -0,
+    where the signs mix it is +0."""
+    P, chunk = 8, 1 << 16
+    comm(P, "double", chunk)
+    count = 200_003
+    xs, outs = _run_special(P, "double", dtype, count, chunk)
+    f = arith.to_float64(outs[3], dtype)
+    cls = inputs.special_class(0, count)
+    sub = cls == 2
+    assert (f[sub] != 0).mean() > 0.9
+    assert (np.abs(f[sub]) < 2.0 ** -126).all()
+    z = cls == 3
+    vals = np.stack([arith.to_float64(x, dtype)[z] for x in xs])
+    all_neg = np.signbit(vals).all(axis=0)
+    assert (f[z] == 0).all()
+    assert np.array_equal(np.signbit(f[z]), all_neg) and all_neg.any() and (~all_neg).any()
+
+
+_R50 = {}
+
+
+def _resnet50_reference(P, kind, chunk):
+    """The oracle's whole-buffer result for the ResNet-50 set (cached per tree kind:
+    B and C1 share it)."""
+    if "xs" not in _R50:
+        ends = workloads.layer_ends("resnet50")
+        _R50["xs"] = [inputs.gradients(r, ends[-1], "float32", layer_ends=ends)
+                      for r in range(P)]
+    if kind not in _R50:
+        _R50[kind] = oar.reference(_R50["xs"], kind, chunk, "float32")[0]
+    return _R50[kind]
+
+
+@pytest.mark.parametrize("kind", ["single", "double", "rotated"])
+@pytest.mark.parametrize("overlap", [True, False])
+def test_full_size_resnet50_fp32_whole_buffer(comm, kind, overlap):
+    """configs[1] at full size in the bench's launch configuration (P = 8, 256 KiB
+    chunks, auto channels): EVERY element of every rank's buffer bit-exact vs the
+    oracle's definition (the whole 25.6M-element fold)."""
+    P, chunk = 8, 256 << 10
+    comm(P, kind, chunk)
+    ends = workloads.layer_ends("resnet50")
+    count = ends[-1]
+    ts = device_inputs(P, count, "float32", layer_ends=ends)
+    ccube.set_overlap(overlap)
+    ccube.allreduce_tree_local(ts)
+    torch.cuda.synchronize()
+    ref = _resnet50_reference(P, kind, chunk)
+    for r in range(P):
+        got = to_numpy(ts[r], "float32")
+        assert np.array_equal(got.view(np.uint32), ref.view(np.uint32)), \
+            f"rank {r}: {int((got.view(np.uint32) != ref.view(np.uint32)).sum())} elements differ"

@@ -50,3 +50,13 @@ def test_workloads_match_torchvision():
             else:
                 groups[-1] += p.numel()
         assert groups == workloads.WORKLOADS[name]
+
+
+def test_zfnet_layers_match_workload_table():
+    """The ZFNet-like net (f4) has the published layer sizes: 8 layers,
+    62,357,608 parameters, and its queue layers are ZFNET_LAYER_ELEMS."""
+    from paper_conf_hpca_sanghoonsk23_b200.gradient_queue import layer_groups
+    m = workloads.zfnet()
+    groups, _ = layer_groups(m)
+    assert [sum(p.numel() for p in g) for g in groups] == workloads.WORKLOADS["zfnet"]
+    assert workloads.total_elems("zfnet") == 62_357_608

@@ -167,3 +167,88 @@ def test_partition_counts():
     assert partition.num_chunks((64 << 20) // 4, 256 << 10, 4) == 256
     nv = workloads.total_elems("vgg16")
     assert partition.num_chunks(nv, 256 << 10, 2) == 1056
+
+
+# ---- the special-value recipe (IEEE corner cases) ----------------------
+
+def _special(P, count, dtype):
+    return [inputs.special(r, count, dtype) for r in range(P)]
+
+
+@pytest.mark.parametrize("P", [2, 3, 4, 8])
+@pytest.mark.parametrize("kind", ["single", "double", "rotated"])
+def test_special_fp32_subnormals_are_summed_exactly(P, kind):
+    """Class 2 (subnormals on every rank, |x| < 2^-129): any order's fp32 sum is
+    exact and subnormal, so the oracle must return the exact integer sum of the
+    mantissas times 2^-149 — a flush-to-zero anywhere would give 0 instead."""
+    count = 6000
+    xs = _special(P, count, "float32")
+    out = allreduce.reference(xs, kind, 1024, "float32")[0]
+    cls = inputs.special_class(0, count)
+    sel = cls == 2
+    bits = np.stack([x.view(np.uint32)[sel] for x in xs]).astype(np.int64)
+    mag = bits & 0x7FFFFFFF
+    sgn = np.where(bits >> 31, -1, 1)
+    exact = (sgn * mag).sum(axis=0)                      # units of 2^-149
+    assert np.array_equal(out[sel].astype(np.float64), np.ldexp(exact.astype(np.float64), -149))
+    assert (out[sel] != 0).sum() > 0.9 * sel.sum()
+    assert (np.abs(out[sel]) < 2.0 ** -126).all()
+
+
+@pytest.mark.parametrize("P", [2, 4, 5, 8])
+@pytest.mark.parametrize("dtype", ["float32", "bfloat16"])
+def test_special_signed_zeros(P, dtype):
+    """Class 3: an IEEE RN sum is -0 only when every addend is -0; with any +0 among
+    them it is +0 (IEEE 754 §6.3).  Both hold per element whatever the tree."""
+    count = 6000
+    xs = _special(P, count, dtype)
+    for kind in ("single", "double"):
+        out = arith.to_float64(allreduce.reference(xs, kind, 1024, dtype)[0], dtype)
+        sel = inputs.special_class(0, count) == 3
+        vals = np.stack([arith.to_float64(x, dtype)[sel] for x in xs])
+        assert (vals == 0).all()
+        all_neg = np.signbit(vals).all(axis=0)
+        assert all_neg.sum() > 50 and (~all_neg).sum() > 50
+        assert (out[sel] == 0).all()
+        assert np.array_equal(np.signbit(out[sel]), all_neg)
+
+
+@pytest.mark.parametrize("P", [2, 4, 6, 8])
+def test_special_fp32_cancellation_gives_plus_zero(P):
+    """Class 6 at even P: +m on even ranks, -m on odd, every partial sum exact, so
+    the exact total is 0 and the RN result is +0 in every tree and order."""
+    count = 6000
+    xs = _special(P, count, "float32")
+    sel = inputs.special_class(0, count) == 6
+    for kind in ("single", "double", "rotated"):
+        out = allreduce.reference(xs, kind, 1024, "float32")[0][sel]
+        assert (out == 0).all() and not np.signbit(out).any()
+
+
+@pytest.mark.parametrize("dtype", ["float32", "bfloat16"])
+def test_special_values_stay_finite_and_within_the_bound(dtype):
+    """Near-max (class 4) sums of 8 cannot overflow; every result obeys the same
+    error bound as the normal recipe (Higham for fp32; per-node rounding for bf16)."""
+    P, count = 8, 8000
+    xs = _special(P, count, dtype)
+    out = arith.to_float64(allreduce.reference(xs, "double", 1024, dtype)[0], dtype)
+    vals = np.stack([arith.to_float64(x, dtype) for x in xs])
+    assert np.isfinite(out).all()
+    s, a = vals.sum(axis=0), np.abs(vals).sum(axis=0)
+    if dtype == "float32":
+        u = 2.0 ** -24
+        g = (P - 1) * u / (1 - (P - 1) * u)
+        # subnormal results carry an absolute error of at most half an ulp of 2^-149
+        assert (np.abs(out - s) <= g * a + 2.0 ** -150).all()
+    else:
+        assert (np.abs(out - s) <= (3 * 2.0 ** -8 + 7 * 2.0 ** -24) * a + 2.0 ** -133).all()
+
+
+def test_special_int32_is_the_wrapped_sum():
+    P, count = 8, 6000
+    xs = _special(P, count, "int32")
+    assert (np.concatenate(xs) == np.iinfo(np.int32).min).any()
+    assert (np.concatenate(xs) == np.iinfo(np.int32).max).any()
+    want = np.sum(np.stack(xs).astype(np.int64), axis=0).astype(np.uint64).astype(np.uint32)
+    for kind in ("single", "double", "rotated"):
+        assert np.array_equal(allreduce.reference(xs, kind, 1024, "int32")[0].view(np.uint32), want)
