@@ -33,7 +33,7 @@ NVLINK_NOMINAL_GBS = 900.0
 NVLINK_MEASURED_GBS = 770.0   # B200_PROFILING.md: measured peer copy per direction
 
 
-def parse():
+def parse(argv=None):
     p = argparse.ArgumentParser()
     p.add_argument("--gpus", type=int, default=1)
     p.add_argument("--steps", type=int, default=200)
@@ -90,12 +90,17 @@ def parse():
     p.add_argument("--cpu-cores", type=int, default=0,
                    help="cpu_baseline: also time the oracle on this many host cores "
                         "(0 = all of them, 1 = skip the all-cores figure)")
-    a = p.parse_args()
+    a = p.parse_args(argv)
     if a.dtype is None:
         a.dtype = "bfloat16" if a.workload == "vgg16" else "float32"
     if a.tree is None:
         a.tree = "double" if a.workload == "vgg16" else "single"
     return a
+
+
+def parse_args_list(argv):
+    """parse() on an explicit argument list (tools reuse bench.py's defaults)."""
+    return parse(argv)
 
 
 def measured_peaks():

@@ -216,6 +216,16 @@ CCUBE_API ccube_result_t ccube_set_threads(int threads);
 #define CCUBE_DATAPATH_TMA 1
 CCUBE_API ccube_result_t ccube_set_datapath(int datapath);
 
+/* Protocol of one-chunk calls (count * elemsize <= chunk_bytes and <= 256 KiB, no
+ * fused update): 1 (default; CCUBE_LL env) = the LL ("low latency") kernel — the
+ * same tree-0 fold in the same order (bitwise the same result), but every 8 bytes
+ * of payload travel with the call's epoch and the consumer polls the data itself,
+ * so a tree hop costs one store-to-load propagation instead of data stores, a
+ * fence, a counter store and a counter poll (eq 3's alpha); the LL lines
+ * are 2x the payload.  0 = the chunked kernel for every size.  Collective with
+ * several processes, like the other settings.  Errors: NOT_INITIALIZED, INVALID_ARG. */
+CCUBE_API ccube_result_t ccube_set_protocol(int ll);
+
 /* Edge transport (physical-topology awareness, cf. §IV).  PUSH: a
  * child stores its partial sum into the parent's receive plane (posted NVLink
  * writes, the default across GPUs).  PULL: the child keeps its partial in place
@@ -284,6 +294,8 @@ typedef struct {
   int last_channels, last_ctas;
   int datapath;                 /* configured CCUBE_DATAPATH_* */
   int last_tma;                 /* 1 = the most recent launch ran the TMA datapath */
+  int protocol;                 /* configured: 1 = LL for one-chunk calls, 0 = off */
+  int last_ll;                  /* 1 = the most recent call ran the LL kernel */
 } ccube_info_t;
 CCUBE_API ccube_result_t ccube_get_info(ccube_info_t *info);
 

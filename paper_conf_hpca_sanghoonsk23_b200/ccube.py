@@ -48,6 +48,7 @@ EXPORTS = [
     "ccube_barrier",
     "ccube_plan_launch",
     "ccube_measure_peer_bandwidth",
+    "ccube_set_protocol",
 ]
 
 
@@ -73,7 +74,8 @@ class Info(ctypes.Structure):
                 ("channels", ctypes.c_int), ("threads", ctypes.c_int), ("overlap", ctypes.c_int),
                 ("transport", ctypes.c_int), ("chunk_bytes", ctypes.c_size_t), ("epoch_base", ctypes.c_uint64 * 2),
                 ("last_channels", ctypes.c_int), ("last_ctas", ctypes.c_int),
-                ("datapath", ctypes.c_int), ("last_tma", ctypes.c_int)]
+                ("datapath", ctypes.c_int), ("last_tma", ctypes.c_int),
+                ("protocol", ctypes.c_int), ("last_ll", ctypes.c_int)]
 
 
 _lib = None
@@ -105,6 +107,7 @@ def lib() -> ctypes.CDLL:
             "ccube_set_trace": [vp, sz],
             "ccube_set_transport": [i],
             "ccube_set_datapath": [i],
+            "ccube_set_protocol": [i],
             "ccube_finalize": [],
             "ccube_get_info": [ctypes.POINTER(Info)],
             "ccube_tree_parents": [i, i, i, ctypes.POINTER(i)],
@@ -337,6 +340,12 @@ def set_datapath(mode: str) -> None:
     """'auto' (default: TMA for the rotated tree set), 'lsu' (register-staged) or 'tma'
     (cp.async.bulk shared-memory ring)."""
     _check(lib().ccube_set_datapath(DATAPATH[mode]), "ccube_set_datapath")
+
+
+def set_protocol(ll: bool) -> None:
+    """True (default): one-chunk calls run the LL (flag-in-data) kernel; False: the
+    chunked kernel for every size.  Same result either way."""
+    _check(lib().ccube_set_protocol(1 if ll else 0), "ccube_set_protocol")
 
 
 def set_trace(trace_tensor, kmax: int) -> None:

@@ -46,7 +46,22 @@ constexpr size_t kFlagBytes =
 // into the child; single-writer monotone u64 like every other counter.
 enum BarrierSlot { kBarArrive0 = 0, kBarArrive1 = 1, kBarRelease = 2, kBarSlots = 3 };
 CCUBE_HD inline size_t barrier_offset(int slot) { return kFlagBytes + slot * kFlagStride; }
-constexpr size_t kWorkspaceBytes = kFlagBytes + kBarSlots * kFlagStride;
+
+// Low-latency (LL) protocol for single-chunk messages (<= kLLMaxBytes and <= one
+// chunk): the data carries its own flag.  A 16-byte LL line is {d0, e, d1, e} —
+// two 4-byte payload words, each paired with the call's epoch e in one 8-byte word
+// (8-byte stores are single-copy atomic), so a reader that sees e twice has the
+// line, with no fence, no counter and no separate flag round trip per hop.
+// Regions per rank, after the barrier counters: the up-lines of child slot 0 and 1
+// (written by the children) and the down-lines (written by the parent), each
+// kLLRegionBytes = 2 x kLLMaxBytes.  Plus one u64 per rank counting finished LL CTAs.
+constexpr size_t kLLMaxBytes = 256u * 1024u;
+constexpr size_t kLLRegionBytes = 2 * kLLMaxBytes;
+enum LLSlot { kLLUp0 = 0, kLLUp1 = 1, kLLDown = 2, kLLSlots = 3 };
+constexpr size_t kLLBase = kFlagBytes + 4096;   // barrier counters live below
+CCUBE_HD inline size_t ll_offset(int slot) { return kLLBase + slot * kLLRegionBytes; }
+constexpr size_t kLLDoneOffset = kLLBase + kLLSlots * kLLRegionBytes;
+constexpr size_t kWorkspaceBytes = kLLDoneOffset + kFlagStride;
 
 enum Dtype { kInt32 = 0, kFloat32 = 1, kBFloat16 = 2 };
 CCUBE_HD inline int elem_size(int dt) { return dt == kBFloat16 ? 2 : 4; }
@@ -109,6 +124,8 @@ struct LaunchArgs {
   int *err;                   // mapped host word; nonzero = abort
   uint64_t *trace;            // optional landing trace
   uint32_t trace_kmax;
+  uint64_t trace_up;          // CCUBE_TRACE_UP: offset (entries) of the reduce-up
+                              // hand-off trace in `trace`, 0 = none
   int l2_hints;               // 1 = per-stream L2 eviction priorities (keep re-read data)
   int sgd;                    // 1 = fused SGD update at landing (fp32 only)
   float sgd_alpha;            // w <- w - sgd_alpha * g
@@ -116,6 +133,8 @@ struct LaunchArgs {
   int elem_size;              // bytes per element (2 or 4)
   int split_control;          // 1 = separate poll and publish warps (warps 0, 1)
   int backoff_ns;             // data warps' readiness-spin back-off (0 = spin)
+  int debug_nodep;            // CCUBE_DEBUG_NODEP: ignore upstream counters (timing
+                              // experiments only — the results are NOT the AllReduce)
 };
 
 // Kernel launcher (tree_allreduce.cu).  Returns a cudaError_t as int.
@@ -132,6 +151,29 @@ struct BarrierRank {
   uint64_t *child_release[kMaxChildren]; // children's release counters
   int nchild;
 };
+// LL kernel (single-chunk messages): per local rank r, `ctas` CTAs.
+struct LLRank {
+  char *buf;                              // own gradient buffer
+  const char *up_in[kMaxChildren];        // own up-line regions (children write)
+  char *up_out;                           // parent's up-line region of my slot, or null
+  const char *down_in;                    // own down-line region (parent writes)
+  char *down_out[kMaxChildren];           // children's down-line regions
+  uint64_t *enq;                          // own Enqueue Semaphore (tree 0, channel 0)
+  uint64_t *done;                         // own finished-CTA counter
+  int nchild;
+};
+struct LLArgs {
+  LLRank r[kMaxRanks];
+  uint64_t count;        // elements
+  uint64_t done_base;    // finished-CTA count of every rank before this call
+  uint64_t enq_value;    // tree 0's Enqueue Semaphore after this call
+  uint32_t epoch;        // LL flag of this call (>= 1)
+  int ctas;              // CTAs per rank
+  int *err;
+  uint64_t timeout_ns;
+};
+int launch_ll(const LLArgs &args, int dtype, bool sys_scope, int nlocal, int threads,
+              void *stream);
 int launch_barrier(const BarrierRank *ranks, int n, uint64_t epoch, int *err,
                    uint64_t timeout_ns, bool sys_scope, void *stream);
 // ccube_measure_peer_bandwidth's copy: src (local) -> every dst (peer), 128-bit.

@@ -173,6 +173,7 @@ struct Comm {
   int split_control = 1;              // CCUBE_SPLIT_CONTROL env: poll and publish warps
   int backoff_ns = 64;                // CCUBE_BACKOFF_NS env: data warps' spin back-off
   int task_order = 0;                 // CCUBE_TASK_ORDER env: block -> task placement
+  int debug_nodep = 0;                // CCUBE_DEBUG_NODEP env: timing experiments only
   bool sgd = false;                 // fused SGD update (f2)
   float sgd_alpha = 0.0f;
   size_t sgd_bytes = 0;
@@ -195,6 +196,10 @@ struct Comm {
   bool use_memop = true;
   bool gate_flush = false;          // memop waits carry CU_STREAM_WAIT_VALUE_FLUSH
   uint64_t bar_epoch = 0;           // ccube_barrier calls so far
+  int ll = 1;                       // CCUBE_LL / ccube_set_protocol: LL for one-chunk calls
+  uint32_t ll_epoch = 0;            // LL calls so far (the flag of the next one is +1)
+  uint64_t ll_done = 0;             // LL CTAs finished per rank so far
+  int last_ll = 0;                  // the most recent call ran the LL kernel
 };
 
 Comm g;
@@ -236,7 +241,10 @@ ccube_result_t check_err_word() {
   if (g.err_host && *reinterpret_cast<volatile int *>(g.err_host) != 0) {
     volatile int *e = g.err_host;
     g.poisoned = true;
-    const char *what = e[0] == 2 ? "gradient-queue gate" : e[0] == 3 ? "barrier" : "AllReduce";
+    const char *what = e[0] == 2   ? "gradient-queue gate"
+                       : e[0] == 3 ? "barrier"
+                       : e[0] == 4 ? "LL AllReduce"
+                                   : "AllReduce";
     return fail(CCUBE_ERR_TIMEOUT,
                 "device watchdog fired in the %s kernel (block %d waited for counter >= %d, "
                 "saw %d); the communicator must be finalized",
@@ -545,6 +553,68 @@ ccube_result_t check_chunk(size_t chunk_bytes) {
   return CCUBE_SUCCESS;
 }
 
+// One-chunk calls on the LL protocol (see tree_allreduce.cu): tree 0 carries the
+// chunk (a3: chunk 0 is on tree 0 for every tree kind), so the result is the chunked
+// path's bit for bit; the epochs of the other trees do not move (K_t = 0).
+ccube_result_t ll_impl(Registration *R, size_t count, ccube_dtype_t dtype, uint64_t E,
+                       void *stream) {
+  const Tree &tr = g.trees[0];
+  LLArgs a;
+  memset(&a, 0, sizeof a);
+  const uint64_t bytes = count * elem_size(dtype);
+  const uint64_t lines = (bytes + 7) / 8;
+  const int threads = 512;
+  uint64_t ctas = (lines + 4 * threads - 1) / (4 * threads);  // <= 4 lines per thread
+  if (ctas > 16) ctas = 16;
+  a.ctas = static_cast<int>(ctas);
+  a.count = count;
+  a.epoch = g.ll_epoch + 1;
+  a.done_base = g.ll_done;
+  a.enq_value = g.base[0] + 1;
+  a.err = g.err_dev;
+  a.timeout_ns = g.timeout_ns;
+  for (int i = 0; i < g.nlocal; ++i) {
+    const int r = g.rank0 + i;
+    LLRank &m = a.r[i];
+    char *own = g.flags_local[i];
+    m.buf = R->bufs[i];
+    m.nchild = tr.nchild[r];
+    for (int s = 0; s < tr.nchild[r]; ++s) {
+      const int c = tr.child[r][s];
+      if (!g.world_flags[c]) return fail(CCUBE_ERR_BOOTSTRAP, "child %d not mapped", c);
+      m.up_in[s] = own + ll_offset(kLLUp0 + s);
+      m.down_out[s] = g.world_flags[c] + ll_offset(kLLDown);
+    }
+    m.down_in = own + ll_offset(kLLDown);
+    const int par = tr.parent[r];
+    if (par >= 0) {
+      if (!g.world_flags[par]) return fail(CCUBE_ERR_BOOTSTRAP, "parent %d not mapped", par);
+      m.up_out = g.world_flags[par] + ll_offset(kLLUp0 + child_slot(tr, par, r));
+    }
+    m.enq = reinterpret_cast<uint64_t *>(own + flag_offset(0, kEnq, 0));
+    m.done = reinterpret_cast<uint64_t *>(own + kLLDoneOffset);
+  }
+  const int rc = launch_ll(a, dtype, g.sys_scope, g.nlocal, threads, stream);
+  if (rc != cudaSuccess)
+    return fail(CCUBE_ERR_CUDA, "LL kernel launch failed: %s",
+                cudaGetErrorString(static_cast<cudaError_t>(rc)));
+  g.ll_epoch += 1;
+  if (ctas > 1) g.ll_done += ctas;   // a single CTA does not count itself
+  g.have_call = true;
+  g.last_E = E;
+  g.last_channels = 1;   // the gate waits on channel 0 of tree 0
+  g.last_sgd = false;
+  g.last_ctas = static_cast<int>(ctas) * g.nlocal;
+  g.last_tma = 0;
+  g.last_ll = 1;
+  for (int t = 0; t < g.ntrees; ++t) {
+    g.last_base[t] = g.base[t];
+    g.last_K[t] = t == 0 ? 1 : 0;
+  }
+  g.base[0] += 1;
+  return CCUBE_SUCCESS;
+}
+
 ccube_result_t allreduce_impl(void *const *bufs, size_t count, ccube_dtype_t dtype,
                               void *stream) {
   if (!g.init) return fail(CCUBE_ERR_NOT_INITIALIZED, "ccube_init has not been called");
@@ -573,6 +643,7 @@ ccube_result_t allreduce_impl(void *const *bufs, size_t count, ccube_dtype_t dty
 
   const uint64_t E = g.chunk_bytes / es;
   const uint64_t K = (count + E - 1) / E;
+  if (g.ll && !g.sgd && K == 1 && bytes <= kLLMaxBytes) return ll_impl(R, count, dtype, E, stream);
   if (K > 0xffffffffull) return fail(CCUBE_ERR_INVALID_ARG, "too many chunks");
 
   // all CTAs spin on each other: they must be co-resident
@@ -622,12 +693,18 @@ ccube_result_t allreduce_impl(void *const *bufs, size_t count, ccube_dtype_t dty
   a.err = g.err_dev;
   a.trace = g.trace;
   a.trace_kmax = static_cast<uint32_t>(g.trace_kmax);
+  // profiling only (tools/pipeline_profile.py): with CCUBE_TRACE_UP=1 the trace
+  // buffer is twice as long and its second half records, per (rank, tree, chunk,
+  // channel), when the reduce-up partial left the rank for its parent
+  if (g.trace && env_int("CCUBE_TRACE_UP", 0))
+    a.trace_up = static_cast<uint64_t>(g.nlocal) * g.ntrees * g.trace_kmax * J;
   a.l2_hints = g.l2_hints;
   a.sgd = g.sgd ? 1 : 0;
   a.sgd_alpha = g.sgd_alpha;
   a.tma = tma;
   a.split_control = g.split_control;
   a.backoff_ns = g.backoff_ns;
+  a.debug_nodep = g.debug_nodep;
   a.elem_size = static_cast<int>(es);
   a.params = R->d_params;
 
@@ -645,6 +722,7 @@ ccube_result_t allreduce_impl(void *const *bufs, size_t count, ccube_dtype_t dty
   g.last_sgd = g.sgd;
   g.last_ctas = tt->n;
   g.last_tma = tma;
+  g.last_ll = 0;
   for (int t = 0; t < g.ntrees; ++t) {
     g.last_base[t] = g.base[t];
     g.last_K[t] = a.K[t];
@@ -741,7 +819,7 @@ struct Hello {
   int32_t channels, threads, datapath, transport, l2_hints, split_control;
   // the launch geometry is computed locally from the occupancy: every GPU must be
   // the same architecture with the same SM count
-  int32_t sm_count, cc_major, cc_minor, pad;
+  int32_t sm_count, cc_major, cc_minor, ll;
   uint64_t chunk_bytes;
   char busid[32];
   int8_t place[CCUBE_MAX_RANKS];  // the placement (R19), identity when none was set
@@ -949,6 +1027,8 @@ ccube_result_t ccube_init(const ccube_world_t *world, ccube_tree_kind_t tree_kin
   g.split_control = env_int("CCUBE_SPLIT_CONTROL", 1) != 0 ? 1 : 0;
   g.task_order = env_int("CCUBE_TASK_ORDER", 0);
   g.backoff_ns = env_int("CCUBE_BACKOFF_NS", 64);
+  g.debug_nodep = env_int("CCUBE_DEBUG_NODEP", 0);
+  g.ll = env_int("CCUBE_LL", 1) != 0 ? 1 : 0;
   g.datapath = env_int("CCUBE_DATAPATH", CCUBE_DATAPATH_AUTO);
   if (g.datapath != CCUBE_DATAPATH_LSU && g.datapath != CCUBE_DATAPATH_TMA)
     g.datapath = CCUBE_DATAPATH_AUTO;
@@ -976,6 +1056,7 @@ ccube_result_t ccube_init(const ccube_world_t *world, ccube_tree_kind_t tree_kin
   mine.transport = g.transport;
   mine.l2_hints = g.l2_hints;
   mine.split_control = g.split_control;
+  mine.ll = g.ll;
   if (cudaDeviceGetAttribute(&mine.sm_count, cudaDevAttrMultiProcessorCount, g.device) !=
           cudaSuccess ||
       cudaDeviceGetAttribute(&mine.cc_major, cudaDevAttrComputeCapabilityMajor, g.device) !=
@@ -1017,12 +1098,13 @@ ccube_result_t ccube_init(const ccube_world_t *world, ccube_tree_kind_t tree_kin
     }
     if (h.channels != mine.channels || h.threads != mine.threads ||
         h.datapath != mine.datapath || h.transport != mine.transport ||
-        h.l2_hints != mine.l2_hints || h.split_control != mine.split_control) {
+        h.l2_hints != mine.l2_hints || h.split_control != mine.split_control ||
+        h.ll != mine.ll) {
       g = Comm();
       return fail(CCUBE_ERR_INVALID_ARG,
                   "ranks disagree on the launch settings (process %d: CCUBE_CHANNELS %d "
                   "CCUBE_THREADS %d CCUBE_DATAPATH %d CCUBE_TRANSPORT %d CCUBE_L2_HINTS %d "
-                  "CCUBE_SPLIT_CONTROL %d; here %d %d %d %d %d %d)",
+                  "CCUBE_SPLIT_CONTROL %d, or CCUBE_LL; here %d %d %d %d %d %d)",
                   p, h.channels, h.threads, h.datapath, h.transport, h.l2_hints,
                   h.split_control, mine.channels, mine.threads, mine.datapath, mine.transport,
                   mine.l2_hints, mine.split_control);
@@ -1315,6 +1397,17 @@ ccube_result_t ccube_set_datapath(int datapath) {
   return CCUBE_SUCCESS;
 }
 
+ccube_result_t ccube_set_protocol(int ll) {
+  std::lock_guard<std::mutex> lk(g_mu);
+  if (!g.init) return fail(CCUBE_ERR_NOT_INITIALIZED, "ccube_init has not been called");
+  const ccube_result_t v = ll != 0 && ll != 1
+                               ? fail(CCUBE_ERR_INVALID_ARG, "protocol must be 0 or 1")
+                               : CCUBE_SUCCESS;
+  CC_TRY(agree_setting("the LL protocol (on/off)", ll, v));
+  g.ll = ll;
+  return CCUBE_SUCCESS;
+}
+
 ccube_result_t ccube_set_transport(int mode) {
   std::lock_guard<std::mutex> lk(g_mu);
   if (!g.init) return fail(CCUBE_ERR_NOT_INITIALIZED, "ccube_init has not been called");
@@ -1384,6 +1477,8 @@ ccube_result_t ccube_get_info(ccube_info_t *info) {
   info->last_ctas = g.last_ctas;
   info->datapath = g.datapath;
   info->last_tma = g.last_tma;
+  info->protocol = g.ll;
+  info->last_ll = g.last_ll;
   return CCUBE_SUCCESS;
 }
 

@@ -220,13 +220,13 @@ struct Combine<kBFloat16> {
 };
 
 __device__ __forceinline__ void trace_landing(const LaunchArgs &a, int local, int t, uint32_t k0,
-                                              uint32_t k1, int j) {
+                                              uint32_t k1, int j, uint64_t base = 0) {
   if (a.trace == nullptr || local < 0) return;
   const uint64_t now = globaltimer();
   for (uint32_t k = k0; k < k1 && k < a.trace_kmax; ++k) {
     const uint64_t idx =
         ((static_cast<uint64_t>(local) * a.ntrees + t) * a.trace_kmax + k) * a.nchannels + j;
-    a.trace[idx] = now;
+    a.trace[base + idx] = now;
   }
 }
 
@@ -482,6 +482,7 @@ __device__ __forceinline__ void publish(const LaunchArgs &a, const TreeParams &p
   if (role == kRoleUpdate) return;
   if (role == kRoleUp && !p.is_root) {
     st_relaxed<SYS>(p.head_out + stride, v);
+    if (a.trace_up) trace_landing(a, p.self_local, t, pub, d, j, a.trace_up);
     return;
   }
   if (role == kRoleUp) {  // root: the chunk is final in my own buffer
@@ -634,7 +635,7 @@ __device__ void poll_warp(const LaunchArgs &a, const TreeParams &p, int role, in
     up = p.enq + stride;
   }
   const bool hold_all = role == kRoleDown && p.is_root;  // B-mode root (Obs #1)
-  uint64_t ready = (role == kRoleUp && p.nchild == 0) ? K : 0;  // a leaf's input is ready
+  uint64_t ready = (role == kRoleUp && p.nchild == 0) || a.debug_nodep ? K : 0;  // a leaf's input is ready
   if (lane == 0) st_release_cta(&sh.ready, ready);
   Watch wd;
   watch_reset(wd);
@@ -1100,6 +1101,175 @@ __global__ void gate_kernel(const GateArgs g) {
   }
 }
 
+// ---- LL protocol: single-chunk messages (latency-bound regime) ------------------
+// The whole message is one chunk of tree 0 (a3: K = 1), so the fold is the same
+// fixed-order tree fold as the chunked path (R2/R3) and the result is bitwise the
+// same.  What changes is the hand-off: instead of data stores, a fence and a
+// counter per hop (three loaded memory round trips), every 8 bytes of payload carry
+// the call's epoch and the consumer polls the data itself (eq 3's alpha term).
+// Phase 1 (reduce-up): per line, own ⊕ child_lo ⊕ child_hi, LL-stored into the
+// parent's up-lines; the root instead writes the final value to its buffer and
+// LL-stores it into its children's down-lines at once (C1 turnaround).
+// Phase 2 (broadcast-down, non-root): wait for the down-line, write the final value
+// to the buffer (the gradient queue), forward it to the children.  The last CTA of a
+// rank publishes its Enqueue Semaphore (a8) so ccube_gradq_wait works unchanged.
+template <bool SYS>
+__device__ __forceinline__ uint4 ll_load(const char *p) {
+  uint4 v;
+  if (SYS)
+    asm volatile("ld.relaxed.sys.global.v4.u32 {%0,%1,%2,%3}, [%4];"
+                 : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p) : "memory");
+  else
+    asm volatile("ld.relaxed.gpu.global.v4.u32 {%0,%1,%2,%3}, [%4];"
+                 : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p) : "memory");
+  return v;
+}
+template <bool SYS>
+__device__ __forceinline__ void ll_store(char *p, uint32_t d0, uint32_t d1, uint32_t e) {
+  if (SYS)
+    asm volatile("st.relaxed.sys.global.v4.u32 [%0], {%1,%2,%3,%4};" ::"l"(p), "r"(d0), "r"(e),
+                 "r"(d1), "r"(e) : "memory");
+  else
+    asm volatile("st.relaxed.gpu.global.v4.u32 [%0], {%1,%2,%3,%4};" ::"l"(p), "r"(d0), "r"(e),
+                 "r"(d1), "r"(e) : "memory");
+}
+
+// Poll an LL line until both of its 8-byte words carry the epoch.
+template <bool SYS>
+__device__ __forceinline__ bool ll_wait(const char *p, uint32_t e, const LLArgs &a, uint64_t &t0,
+                                        uint32_t &d0, uint32_t &d1) {
+  uint32_t spins = 0;
+  for (;;) {
+    const uint4 v = ll_load<SYS>(p);
+    if (v.y == e && v.w == e) {
+      d0 = v.x;
+      d1 = v.z;
+      return true;
+    }
+    if ((++spins & 255) == 0) {
+      const uint64_t now = globaltimer();
+      if (t0 == 0) t0 = now;
+      if (*reinterpret_cast<volatile int *>(a.err) != 0) return false;
+      if (now - t0 > a.timeout_ns) {
+        volatile int *err = reinterpret_cast<volatile int *>(a.err);
+        err[1] = static_cast<int>(blockIdx.x);
+        err[2] = static_cast<int>(e);
+        err[3] = static_cast<int>(v.y);
+        __threadfence_system();
+        err[0] = 4;  // 4 = LL watchdog
+        __threadfence_system();
+        return false;
+      }
+    }
+  }
+}
+
+// One node's combine on a word pair: own, then each child's partial in ascending
+// rank, left to right (R2); bf16 accumulates both halves in fp32 and rounds once
+// per node output (R3); a leaf's own bits are forwarded untouched.
+template <int DT>
+__device__ __forceinline__ uint32_t ll_combine(uint32_t own, const uint32_t *c, int n) {
+  if (n == 0) return own;
+  if (DT == kInt32) {
+    for (int i = 0; i < n; ++i) own += c[i];
+    return own;
+  } else if (DT == kFloat32) {
+    float f = __uint_as_float(own);
+    for (int i = 0; i < n; ++i) f = __fadd_rn(f, __uint_as_float(c[i]));
+    return __float_as_uint(f);
+  } else {
+    float lo = bf_lo(own), hi = bf_hi(own);
+    for (int i = 0; i < n; ++i) {
+      lo = __fadd_rn(lo, bf_lo(c[i]));
+      hi = __fadd_rn(hi, bf_hi(c[i]));
+    }
+    return bf_round(lo) | (bf_round(hi) << 16);
+  }
+}
+
+// Guarded access to payload word w (4 bytes) of a buffer of `nbytes` bytes: the
+// last word of an odd-length bf16 buffer holds one element.
+__device__ __forceinline__ uint32_t ll_get(const char *buf, uint64_t w, uint64_t nbytes) {
+  const uint64_t o = 4 * w;
+  if (o + 4 <= nbytes) return *reinterpret_cast<const uint32_t *>(buf + o);
+  if (o + 2 <= nbytes) return *reinterpret_cast<const uint16_t *>(buf + o);
+  return 0;
+}
+__device__ __forceinline__ void ll_put(char *buf, uint64_t w, uint64_t nbytes, uint32_t v) {
+  const uint64_t o = 4 * w;
+  if (o + 4 <= nbytes)
+    *reinterpret_cast<uint32_t *>(buf + o) = v;
+  else if (o + 2 <= nbytes)
+    *reinterpret_cast<uint16_t *>(buf + o) = static_cast<uint16_t>(v);
+}
+
+template <int DT, bool SYS>
+__global__ void __launch_bounds__(512) ll_kernel(const LLArgs a) {
+  const int rank = blockIdx.x / a.ctas;
+  const int part = blockIdx.x % a.ctas;
+  const LLRank &me = a.r[rank];
+  const uint64_t nbytes = a.count * (DT == kBFloat16 ? 2 : 4);
+  const uint64_t lines = (nbytes + 7) / 8;  // 8 payload bytes per 16-byte line
+  const uint64_t stride = static_cast<uint64_t>(a.ctas) * blockDim.x;
+  const uint32_t e = a.epoch;
+  uint64_t t0 = 0;
+  bool ok = true;
+  // phase 1: reduce-up (and the root's turnaround)
+  for (uint64_t l = static_cast<uint64_t>(part) * blockDim.x + threadIdx.x; l < lines && ok;
+       l += stride) {
+    uint32_t w0 = ll_get(me.buf, 2 * l, nbytes), w1 = ll_get(me.buf, 2 * l + 1, nbytes);
+    uint32_t c0[kMaxChildren], c1[kMaxChildren];
+    for (int s = 0; s < me.nchild && ok; ++s)
+      ok = ll_wait<SYS>(me.up_in[s] + 16 * l, e, a, t0, c0[s], c1[s]);
+    if (!ok) break;
+    w0 = ll_combine<DT>(w0, c0, me.nchild);
+    w1 = ll_combine<DT>(w1, c1, me.nchild);
+    if (me.up_out) {
+      ll_store<SYS>(me.up_out + 16 * l, w0, w1, e);
+    } else {  // root: final
+      ll_put(me.buf, 2 * l, nbytes, w0);
+      ll_put(me.buf, 2 * l + 1, nbytes, w1);
+      for (int s = 0; s < me.nchild; ++s) ll_store<SYS>(me.down_out[s] + 16 * l, w0, w1, e);
+    }
+  }
+  // phase 2: broadcast-down
+  if (me.up_out) {
+    for (uint64_t l = static_cast<uint64_t>(part) * blockDim.x + threadIdx.x; l < lines && ok;
+         l += stride) {
+      uint32_t w0, w1;
+      ok = ll_wait<SYS>(me.down_in + 16 * l, e, a, t0, w0, w1);
+      if (!ok) break;
+      ll_put(me.buf, 2 * l, nbytes, w0);
+      ll_put(me.buf, 2 * l + 1, nbytes, w1);
+      for (int s = 0; s < me.nchild; ++s) ll_store<SYS>(me.down_out[s] + 16 * l, w0, w1, e);
+    }
+  }
+  // the rank's last CTA to finish publishes the Enqueue Semaphore: every final word
+  // of this rank is in its buffer (the gradient-queue gate's condition, a8/a9)
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    fence_release<SYS>();
+    if (a.ctas == 1) {  // the only CTA of the rank: no count to take
+      st_relaxed<SYS>(me.enq, ok ? a.enq_value : ~0ull);
+      return;
+    }
+    const unsigned long long prev = atomicAdd(reinterpret_cast<unsigned long long *>(me.done), 1ull);
+    if (prev + 1 == a.done_base + a.ctas) {
+      fence_release<SYS>();
+      st_relaxed<SYS>(me.enq, ok ? a.enq_value : ~0ull);
+    }
+  }
+}
+
+template <int DT>
+int launch_ll_t(const LLArgs &a, bool sys_scope, int nlocal, int threads, cudaStream_t s) {
+  if (sys_scope)
+    ll_kernel<DT, true><<<nlocal * a.ctas, threads, 0, s>>>(a);
+  else
+    ll_kernel<DT, false><<<nlocal * a.ctas, threads, 0, s>>>(a);
+  return static_cast<int>(cudaGetLastError());
+}
+
 // Device-side barrier over tree 0 (ccube_barrier): warp i serves local rank i.
 // Lane s < nchild waits for child s's "arrive" >= epoch; then lane 0 tells the
 // parent (release store into the parent's counter), waits for the parent's
@@ -1242,6 +1412,19 @@ int launch_gate(const uint64_t *const *counters, const uint64_t *targets, int n,
   else
     gate_kernel<false><<<1, 32, 0, s>>>(g);
   return static_cast<int>(cudaGetLastError());
+}
+
+int launch_ll(const LLArgs &args, int dtype, bool sys_scope, int nlocal, int threads,
+              void *stream) {
+  if (nlocal < 1 || nlocal > kMaxRanks || args.ctas < 1 || threads < 32 || threads > 512)
+    return cudaErrorInvalidValue;
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  switch (dtype) {
+    case kInt32: return launch_ll_t<kInt32>(args, sys_scope, nlocal, threads, s);
+    case kFloat32: return launch_ll_t<kFloat32>(args, sys_scope, nlocal, threads, s);
+    case kBFloat16: return launch_ll_t<kBFloat16>(args, sys_scope, nlocal, threads, s);
+    default: return cudaErrorInvalidValue;
+  }
 }
 
 int launch_barrier(const BarrierRank *ranks, int n, uint64_t epoch, int *err,

@@ -37,9 +37,7 @@ def measure_peer_bandwidth(pg=None, nbytes: int = 64 << 20, reps: int = 3):
         finally:
             ccube.finalize()
         return pair
-    dev = torch.device("cuda", torch.cuda.current_device()) if on_gpu else torch.device("cpu")
-    buf = torch.empty(nbytes // 4, dtype=torch.float32, device=dev)
-    sync = torch.cuda.synchronize if on_gpu else (lambda: None)
+    buf = torch.empty(nbytes // 4, dtype=torch.float32)
     bw = torch.zeros(P, P, dtype=torch.float64)
     for i in range(P):
         for j in range(P):
@@ -48,20 +46,17 @@ def measure_peer_bandwidth(pg=None, nbytes: int = 64 << 20, reps: int = 3):
             dist.barrier(group=pg)
             best = float("inf")
             for _ in range(reps):
-                sync()
                 t0 = time.perf_counter()
                 if me == i:
                     dist.send(buf, dst=dist.get_global_rank(pg, j), group=pg)
                 elif me == j:
                     dist.recv(buf, src=dist.get_global_rank(pg, i), group=pg)
-                sync()
                 best = min(best, time.perf_counter() - t0)
             if me == j:
                 bw[i, j] = nbytes / best / 1e9
     # the receiver's number is authoritative; share it with everyone
-    t = bw.to(dev)
-    dist.all_reduce(t, op=dist.ReduceOp.SUM, group=pg)
-    return t.cpu().tolist()
+    dist.all_reduce(bw, op=dist.ReduceOp.SUM, group=pg)
+    return bw.tolist()
 
 
 def plan(pg=None, kind: str = "double", **measure_kw):

@@ -664,3 +664,77 @@ def test_full_size_resnet50_fp32_whole_buffer(comm, kind, overlap):
         got = to_numpy(ts[r], "float32")
         assert np.array_equal(got.view(np.uint32), ref.view(np.uint32)), \
             f"rank {r}: {int((got.view(np.uint32) != ref.view(np.uint32)).sum())} elements differ"
+
+
+# ---- LL protocol (one-chunk calls: flag-in-data) -------------------------
+@pytest.mark.parametrize("P", [2, 3, 4, 5, 8])
+@pytest.mark.parametrize("kind", ["single", "double", "rotated"])
+@pytest.mark.parametrize("dtype", ["int32", "float32", "bfloat16"])
+@pytest.mark.parametrize("count", [1, 3, 1023, 20_001])
+def test_parity_ll(comm, P, kind, dtype, count):
+    """A one-chunk message runs the LL kernel: bit-exact vs the oracle (tree 0's fold)
+    for every tree kind, odd bf16 counts included."""
+    chunk = 256 << 10
+    comm(P, kind, chunk)
+    xs, outs = _run(P, kind, dtype, count, chunk)
+    assert ccube.get_info()["last_ll"] == 1
+    ref = oar.reference(xs, kind, chunk, dtype)[0]
+    for r in range(P):
+        assert np.array_equal(outs[r], ref), f"rank {r}"
+
+
+@pytest.mark.parametrize("dtype", ["float32", "bfloat16"])
+def test_ll_special_values_and_max_size(comm, dtype):
+    """IEEE corner cases through the LL kernel, at its largest message (256 KiB)."""
+    P, chunk = 8, 256 << 10
+    comm(P, "double", chunk)
+    count = (256 << 10) // arith.ELEM_SIZE[dtype]
+    xs, outs = _run_special(P, "double", dtype, count, chunk)
+    assert ccube.get_info()["last_ll"] == 1
+    ref = oar.reference(xs, "double", chunk, dtype)[0]
+    for r in range(P):
+        assert np.array_equal(outs[r], ref), f"rank {r}"
+
+
+def test_ll_equals_chunked_and_interleaves(comm):
+    """LL and chunked calls alternate on one communicator (epochs and counters stay
+    consistent); both give the same bits as the oracle; LL off runs the chunked
+    kernel for the same one-chunk size."""
+    P, chunk = 8, 64 << 10
+    comm(P, "double", chunk)
+    for it, count in enumerate([100, 50_000, 7, 16_384, 70_001, 1]):
+        ccube.set_protocol(it % 3 != 2)
+        xs, outs = _run(P, "double", "float32", count, chunk, seed=300 + it)
+        ll = count * 4 <= chunk and it % 3 != 2
+        assert ccube.get_info()["last_ll"] == int(ll), (it, count)
+        ref = oar.reference(xs, "double", chunk, "float32")[0]
+        for r in range(P):
+            assert np.array_equal(outs[r], ref), (it, r)
+
+
+def test_ll_gate_opens_after_landing(comm):
+    """ccube_gradq_wait after an LL call: every layer's snapshot holds final values."""
+    P, chunk = 8, 256 << 10
+    comm(P, "single", chunk)
+    count = 60_000
+    ends = [1000, 30_000, count]
+    ts = device_inputs(P, count, "float32")
+    ccube.gradq_set_layers(ends)
+    cs, comp = torch.cuda.Stream(), torch.cuda.Stream()
+    cs.wait_stream(torch.cuda.current_stream())
+    comp.wait_stream(torch.cuda.current_stream())
+    with torch.cuda.stream(cs):
+        ccube.allreduce_tree_local(ts, stream=cs)
+    snaps = []
+    with torch.cuda.stream(comp):
+        lo = 0
+        for l, hi in enumerate(ends):
+            ccube.gradq_wait_local(7, l, stream=comp)
+            snaps.append(ts[7][lo:hi].clone())
+            lo = hi
+    torch.cuda.synchronize()
+    assert ccube.get_info()["last_ll"] == 1
+    lo = 0
+    for s, hi in zip(snaps, ends):
+        assert torch.equal(s, ts[7][lo:hi])
+        lo = hi
