@@ -199,8 +199,9 @@ CCUBE_API ccube_result_t ccube_set_overlap(int on);
  * every tree, and the capacity the minimum over GPUs — capped at one channel per
  * two 2 KB units of a chunk, or per unit for buffers of >= 16 chunks).  Both ends of
  * an edge therefore always slice chunks alike.  `threads` = data threads per CTA
- * (32..256, multiple of 32; CCUBE_THREADS env, default 256); each CTA adds two
- * control warps. */
+ * (32..256, multiple of 32; CCUBE_THREADS env, default 192 = 6 data warps); each
+ * CTA adds two control warps.  Smaller CTAs give each thread more registers
+ * (two CTAs per SM), which the combines spend on more loads in flight. */
 CCUBE_API ccube_result_t ccube_set_channels(int channels);
 CCUBE_API ccube_result_t ccube_set_threads(int threads);
 

@@ -41,16 +41,19 @@ def _stale() -> bool:
     return any(os.path.getmtime(d) > t for d in deps)
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    if not force and not _stale():
+def build(force: bool = False, verbose: bool = False, target: str = LIB, defines=()) -> str:
+    """Compile and link the library.  ``target`` / ``defines`` (-D macros) build
+    experiment variants (tools/experiments); the product is the default in-tree LIB."""
+    if target == LIB and not defines and not force and not _stale():
         return LIB
     objs = []
-    tmp = os.path.join(HERE, "build")
+    tmp = os.path.join(HERE, "build", os.path.basename(target).replace(".so", ""))
     os.makedirs(tmp, exist_ok=True)
     for src in SOURCES:
         obj = os.path.join(tmp, os.path.splitext(src)[0] + ".o")
         lang = [] if src.endswith(".cu") else ["-x", "cu"]
-        cmd = [nvcc(), *ARCH, *NVCC_FLAGS, "-I", INCLUDE, "-I", CSRC, *lang, "-c",
+        cmd = [nvcc(), *ARCH, *NVCC_FLAGS, *[f"-D{d}" for d in defines], "-I", INCLUDE,
+               "-I", CSRC, *lang, "-c",
                os.path.join(CSRC, src), "-o", obj]
         out = subprocess.run(cmd, capture_output=True, text=True)
         if out.returncode != 0:
@@ -58,14 +61,14 @@ def build(force: bool = False, verbose: bool = False) -> str:
         if verbose:
             sys.stderr.write(out.stderr)
         objs.append(obj)
-    cmd = [nvcc(), *ARCH, "-shared", "-cudart", "static", "-o", LIB + ".tmp", *objs,
+    cmd = [nvcc(), *ARCH, "-shared", "-cudart", "static", "-o", target + ".tmp", *objs,
            "-Xlinker", "--version-script=" + os.path.join(CSRC, "ccube.map"),
            "-lpthread", "-ldl", "-lrt"]
     out = subprocess.run(cmd, capture_output=True, text=True)
     if out.returncode != 0:
         raise RuntimeError(f"link failed:\n{out.stdout}\n{out.stderr}")
-    os.replace(LIB + ".tmp", LIB)
-    return LIB
+    os.replace(target + ".tmp", target)
+    return target
 
 
 if __name__ == "__main__":

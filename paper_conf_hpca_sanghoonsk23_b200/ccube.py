@@ -86,10 +86,13 @@ def lib() -> ctypes.CDLL:
     """Load libccube.so (built in-tree by __graft_entry__.build()).  Raises if absent."""
     global _lib
     if _lib is None:
-        if not os.path.exists(LIB_PATH):
-            raise RuntimeError(f"{LIB_PATH} is missing: run `python -m "
+        # CCUBE_LIB: an experiment build of the same sources (tools/experiments); the
+        # product, tests and smoke use the in-tree library
+        path = os.environ.get("CCUBE_LIB") or LIB_PATH
+        if not os.path.exists(path):
+            raise RuntimeError(f"{path} is missing: run `python -m "
                                "paper_conf_hpca_sanghoonsk23_b200.build` (no CPU fallback)")
-        L = ctypes.CDLL(LIB_PATH)
+        L = ctypes.CDLL(path)
         vp, sz, i = ctypes.c_void_p, ctypes.c_size_t, ctypes.c_int
         sig = {
             "ccube_init": [ctypes.POINTER(World), i, sz],

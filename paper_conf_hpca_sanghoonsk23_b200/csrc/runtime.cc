@@ -158,7 +158,10 @@ struct Comm {
   int ntrees = 1;
   size_t chunk_bytes = CCUBE_DEFAULT_CHUNK_BYTES;
   Tree trees[kMaxTrees];
-  int channels = 0, threads = 256, overlap = 1;  // channels 0 = auto
+  // channels 0 = auto; threads = data threads per CTA: 6 data warps (192) + 2
+  // control warps = 256-thread CTAs, 128 registers per thread at two CTAs per SM,
+  // 6 vectors per lane and source in flight in the combines (measured)
+  int channels = 0, threads = kDefaultDataThreads, overlap = 1;
   int tree_kind = CCUBE_TREE_SINGLE;
   uint64_t base[kMaxTrees] = {};
   bool have_call = false;
@@ -1000,7 +1003,7 @@ ccube_result_t ccube_init(const ccube_world_t *world, ccube_tree_kind_t tree_kin
   if (channels < 0 || channels > CCUBE_MAX_CHANNELS)
     return fail(CCUBE_ERR_INVALID_ARG, "CCUBE_CHANNELS %d out of range", channels);
   CC_TRY(check_chunk(chunk_bytes));
-  int threads = env_int("CCUBE_THREADS", 256);
+  int threads = env_int("CCUBE_THREADS", kDefaultDataThreads);
   if (threads < 32 || threads > 256 || threads % 32)
     return fail(CCUBE_ERR_INVALID_ARG, "CCUBE_THREADS %d out of range [32, 256]", threads);
   const int transport = env_int("CCUBE_TRANSPORT", CCUBE_TRANSPORT_AUTO);

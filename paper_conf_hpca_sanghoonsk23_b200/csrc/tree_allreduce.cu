@@ -42,6 +42,28 @@ namespace {
 #ifndef CCUBE_U_COPY
 #define CCUBE_U_COPY 4     // ... (copies; 8 measured 1% slower, v16)
 #endif
+// Smaller CTAs leave each thread more registers at two CTAs per SM (launch bounds:
+// 320 threads -> 96, 256 -> 128, 224 -> 144, 192 -> 168), i.e. room for more
+// 16-byte vectors in flight per lane in the combines (the DRAM-reading UP tasks,
+// whose bytes in flight set the pipeline's rate).  Per CTA-size bucket:
+#ifndef CCUBE_U_COMBINE_S
+#define CCUBE_U_COMBINE_S 6    // <= 256 threads (6 data warps + 2 control warps)
+#endif
+#ifndef CCUBE_U_COMBINE_224
+#define CCUBE_U_COMBINE_224 8  // <= 224 threads (5 data warps)
+#endif
+#ifndef CCUBE_U_COMBINE_192
+#define CCUBE_U_COMBINE_192 8  // <= 192 threads (4 data warps)
+#endif
+#ifndef CCUBE_U_COPY_S
+#define CCUBE_U_COPY_S 4
+#endif
+__host__ __device__ constexpr int u_combine(int maxt) {
+  return maxt <= 192 ? CCUBE_U_COMBINE_192
+         : maxt <= 224 ? CCUBE_U_COMBINE_224
+         : maxt <= 256 ? CCUBE_U_COMBINE_S
+                       : CCUBE_U_COMBINE;
+}
 
 constexpr int kMaxThreads = 320;  // up to 8 data warps + one or two control warps
 constexpr int kMaxDataWarps = 8;
@@ -792,11 +814,11 @@ __device__ void lsu_stream(const LaunchArgs &a, const Endpoints &e, int t, int j
   }
 }
 
-template <int DT, int NIN, bool SGD>
+template <int DT, int NIN, bool SGD, int MAXT>
 __device__ __forceinline__ void lsu_nout(const LaunchArgs &a, const Endpoints &e, int t, int j,
                                          int w, int W, Shared &sh) {
   // block = 2 KB (copies and combines); build-time overrides for experiments
-  constexpr int U = NIN == 1 ? CCUBE_U_COPY : CCUBE_U_COMBINE;
+  constexpr int U = NIN == 1 ? (MAXT <= 256 ? CCUBE_U_COPY_S : CCUBE_U_COPY) : u_combine(MAXT);
   if constexpr (SGD && DT == kFloat32 && NIN <= 2) {
     if (e.sgd) {  // root UP (NIN 2), interior DOWN and leaf UPDATE (NIN 1); U = 4 (2 KB)
       switch (e.nout) {
@@ -1017,7 +1039,7 @@ __device__ void tma_data_warp(const LaunchArgs &a, const TreeParams &p, int role
   }
 }
 
-template <int DT, bool SGD>
+template <int DT, bool SGD, int MAXT>
 __device__ void data_warp(const LaunchArgs &a, const TreeParams &p, int role, int t, int j,
                           int w, int W, Shared &sh) {
   Endpoints e = endpoints(a, p, role);
@@ -1027,9 +1049,9 @@ __device__ void data_warp(const LaunchArgs &a, const TreeParams &p, int role, in
     return;
   }
   switch (e.nin) {
-    case 1: lsu_nout<DT, 1, SGD>(a, e, t, j, w, W, sh); break;
-    case 2: lsu_nout<DT, 2, SGD>(a, e, t, j, w, W, sh); break;
-    default: lsu_nout<DT, 3, SGD>(a, e, t, j, w, W, sh); break;
+    case 1: lsu_nout<DT, 1, SGD, MAXT>(a, e, t, j, w, W, sh); break;
+    case 2: lsu_nout<DT, 2, SGD, MAXT>(a, e, t, j, w, W, sh); break;
+    default: lsu_nout<DT, 3, SGD, MAXT>(a, e, t, j, w, W, sh); break;
   }
 }
 
@@ -1073,7 +1095,7 @@ __global__ void __launch_bounds__(MAXT, kMinBlocksPerSm) tree_allreduce_kernel(c
   } else if (a.tma) {
     tma_data_warp<DT, SGD>(a, p, task.role, task.tree, task.channel, warp - nctl, W, sh, tma_ring);
   } else {
-    data_warp<DT, SGD>(a, p, task.role, task.tree, task.channel, warp - nctl, W, sh);
+    data_warp<DT, SGD, MAXT>(a, p, task.role, task.tree, task.channel, warp - nctl, W, sh);
   }
 }
 
@@ -1343,26 +1365,28 @@ __global__ void __launch_bounds__(256) peer_copy_kernel(const PeerCopyArgs c) {
   }
 }
 
+// The kernel instance for a CTA of `threads` threads: the smallest size bucket
+// (192 / 224 / 256 / 320) that holds it.
+template <int DT, bool SYS, bool SGD>
+void (*kernel_for(int threads))(const LaunchArgs) {
+  if (threads <= 192) return tree_allreduce_kernel<DT, SYS, SGD, 192>;
+  if (threads <= 224) return tree_allreduce_kernel<DT, SYS, SGD, 224>;
+  if (threads <= 256) return tree_allreduce_kernel<DT, SYS, SGD, 256>;
+  return tree_allreduce_kernel<DT, SYS, SGD, kMaxThreads>;
+}
+
 template <int DT, bool SYS, bool SGD>
 int launch_t(const LaunchArgs &a, int grid, int threads, cudaStream_t s) {
   const size_t smem = a.tma ? kTmaRing : 0;
-  if (threads <= 256) {
-    auto *fn = tree_allreduce_kernel<DT, SYS, SGD, 256>;
-    if (smem) cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-    fn<<<grid, threads, smem, s>>>(a);
-  } else {
-    auto *fn = tree_allreduce_kernel<DT, SYS, SGD, kMaxThreads>;
-    if (smem) cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-    fn<<<grid, threads, smem, s>>>(a);
-  }
+  auto *fn = kernel_for<DT, SYS, SGD>(threads);
+  if (smem) cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  fn<<<grid, threads, smem, s>>>(a);
   return static_cast<int>(cudaGetLastError());
 }
 
 template <int DT, bool SYS, bool SGD>
 const void *kernel_ptr(int threads) {
-  if (threads <= 256)
-    return reinterpret_cast<const void *>(tree_allreduce_kernel<DT, SYS, SGD, 256>);
-  return reinterpret_cast<const void *>(tree_allreduce_kernel<DT, SYS, SGD, kMaxThreads>);
+  return reinterpret_cast<const void *>(kernel_for<DT, SYS, SGD>(threads));
 }
 
 }  // namespace
