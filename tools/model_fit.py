@@ -69,7 +69,11 @@ def eq7_us(P, N, alpha, beta, coef=3.0):   # C1; coef 2*sqrt(2) = exact
 
 
 def main(path):
-    rows = [json.loads(l) for l in open(path) if l.startswith("{")]
+    allrows = [json.loads(l) for l in open(path) if l.startswith("{")]
+    # the model describes the chunked kernel; the LL kernel's one-chunk latencies are
+    # reported next to it (LL = eq 3's alpha with the flag carried in the data)
+    rows = [r for r in allrows if r.get("protocol", "chunked") == "chunked"]
+    ll = [r for r in allrows if r.get("protocol") == "ll"]
     # 1. t0 and alpha from the one-chunk latency vs hop count
     small = min(r["bytes"] for r in rows)
     pts = [(2 * DEPTH[r["P"]], r["us"]) for r in rows
@@ -80,6 +84,13 @@ def main(path):
     out = {"source": path, "anchor_bytes": small, "t0_us": float(t0), "alpha_us_per_hop": float(alpha),
            "anchor_points": [{"hops": h, "us": t} for h, t in pts],
            "anchor_max_rel_err": float(np.max(np.abs(A @ [t0, alpha] - y) / y)), "fits": []}
+    if ll:
+        lp = [(2 * DEPTH[r["P"]], r["us"]) for r in ll
+              if r["bytes"] == small and r["mode"] == "C1" and r["P"] > 1]
+        A2 = np.array([[1.0, h] for h, _ in lp])
+        (t0_ll, alpha_ll), _ = nnls(A2, np.array([t for _, t in lp]))
+        out["ll"] = {"t0_us": float(t0_ll), "alpha_us_per_hop": float(alpha_ll),
+                     "anchor_points": [{"hops": h, "us": t} for h, t in lp]}
     groups = defaultdict(list)
     for r in rows:
         groups[(r["P"], r["tree"])].append(r)
