@@ -160,6 +160,47 @@ class ClockSampler:
                 "reasons": reasons, "samples": len(rows)}
 
 
+# ------------------------------------------------------------- NVLink counters
+class NvlinkCounters:
+    """NVLink data bytes this GPU sent / received, from NVML's cumulative per-link
+    counters (NVML_FI_DEV_NVLINK_THROUGHPUT_DATA_TX / _RX, KiB; summed over links).
+    Read before and after the timed region at N > 1; unlike an ncu pass it does not
+    serialise the ranks' kernels.  Any failure (no NVML, no NVLink) gives None."""
+
+    LINKS = 18   # NVLink 5 links per B200
+
+    def __init__(self, device_index):
+        self.h = None
+        try:
+            import pynvml as nv
+            import torch
+            nv.nvmlInit()
+            pr = torch.cuda.get_device_properties(device_index)
+            bus = f"{pr.pci_domain_id:08x}:{pr.pci_bus_id:02x}:{pr.pci_device_id:02x}.0"
+            try:
+                self.h = nv.nvmlDeviceGetHandleByPciBusId_v2(bus.encode())
+            except Exception:  # noqa: BLE001
+                self.h = nv.nvmlDeviceGetHandleByIndex(device_index)
+            self.nv = nv
+        except Exception:  # noqa: BLE001
+            self.h = None
+
+    def read(self):
+        """(tx_bytes, rx_bytes) cumulative, or None."""
+        if self.h is None:
+            return None
+        nv = self.nv
+        try:
+            ids = [(nv.NVML_FI_DEV_NVLINK_THROUGHPUT_DATA_TX, l) for l in range(self.LINKS)] + \
+                  [(nv.NVML_FI_DEV_NVLINK_THROUGHPUT_DATA_RX, l) for l in range(self.LINKS)]
+            vals = nv.nvmlDeviceGetFieldValues(self.h, ids)
+            tx = sum(v.value.ullVal for v in vals[:self.LINKS] if v.nvmlReturn == 0)
+            rx = sum(v.value.ullVal for v in vals[self.LINKS:] if v.nvmlReturn == 0)
+            return tx * 1024, rx * 1024
+        except Exception:  # noqa: BLE001
+            return None
+
+
 # ---------------------------------------------------------------- oracle timing
 def oracle_inputs(P, dtype, workload, chunk_bytes, nchunks):
     """Every rank's seeded gradients for the first ``nchunks`` chunks of the workload."""
@@ -507,10 +548,26 @@ def run_ccube(a):
         return restore
 
     clocks = ClockSampler(local_rank if multi else 0, enabled=(rank == 0 and not a.no_clocks))
+    nvl = NvlinkCounters(torch.cuda.current_device()) if multi else None
     time.sleep(0.3)
+    nvl0, t_nvl0 = (nvl.read(), time.perf_counter()) if nvl else (None, 0)
     ms, total_ms = _time_steps(lambda: allreduce(bufs), restorer(bufs, pristine), a.steps,
                                a.warmup, stream, multi, hdev)
+    nvl1, t_nvl1 = (nvl.read(), time.perf_counter()) if nvl else (None, 0)
     clk = clocks.stop()
+    nvlink = None
+    if nvl0 is not None and nvl1 is not None:
+        # the reads bracket the warm-up and the timed steps: one AllReduce each (the
+        # restore copies are local, so every NVLink byte is the AllReduce's)
+        calls = a.steps + max(3, a.warmup)
+        tx, rx = (nvl1[0] - nvl0[0]) / calls, (nvl1[1] - nvl0[1]) / calls
+        t_call = total_ms / a.steps / 1e3
+        nvlink = {"tx_bytes_per_call": tx, "rx_bytes_per_call": rx,
+                  "tx_gbs": tx / t_call / 1e9, "rx_gbs": rx / t_call / 1e9,
+                  "algorithmic_port_bytes": max(_port_loads(P, a.tree)) * nbytes,
+                  "source": "NVML NVLINK_THROUGHPUT_DATA_TX/RX of rank 0's GPU, summed over "
+                            "links, read around warm-up + timed steps; GB/s = bytes per call / "
+                            "device time per call"}
     ms_step = total_ms / a.steps
     bw, alg = busbw(nbytes, ms_step / 1e3, P)
 
@@ -686,7 +743,7 @@ def run_ccube(a):
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
             "dtype": _dt(a.dtype), "data": "synthetic",
             "config": dict(_config(a, P, nbytes), channels=info["last_channels"],
-                           ctas=info["last_ctas"], threads=info["threads"],
+                           ctas=info["last_ctas"], threads=info["last_threads"],
                            datapath="tma" if info["last_tma"] else "lsu",
                            l2=("inputs (P x bytes_per_rank) larger than L2 and restored from a "
                                "pristine copy between timed steps (flushes L2)") if not multi
@@ -702,6 +759,7 @@ def run_ccube(a):
         }
         if multi:
             line["busbw_frac_of_900"] = bw / NVLINK_NOMINAL_GBS
+            line["nvlink_counters_rank0"] = nvlink
             line["result_checksums"] = hashes
             line["port_peak"] = port_peak
         if oracle_check is not None:

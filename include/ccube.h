@@ -199,9 +199,10 @@ CCUBE_API ccube_result_t ccube_set_overlap(int on);
  * every tree, and the capacity the minimum over GPUs — capped at one channel per
  * two 2 KB units of a chunk, or per unit for buffers of >= 16 chunks).  Both ends of
  * an edge therefore always slice chunks alike.  `threads` = data threads per CTA
- * (32..256, multiple of 32; CCUBE_THREADS env, default 192 = 6 data warps); each
- * CTA adds two control warps.  Smaller CTAs give each thread more registers
- * (two CTAs per SM), which the combines spend on more loads in flight. */
+ * (32..256, multiple of 32; 0 = auto, the default; CCUBE_THREADS env); each CTA
+ * adds two control warps.  Smaller CTAs give each thread more registers (two CTAs
+ * per SM), which the combines spend on more loads in flight; auto takes 6 data
+ * warps when each channel's slice of a chunk holds >= 3 units of 2 KB, else 8. */
 CCUBE_API ccube_result_t ccube_set_channels(int channels);
 CCUBE_API ccube_result_t ccube_set_threads(int threads);
 
@@ -297,6 +298,7 @@ typedef struct {
   int last_tma;                 /* 1 = the most recent launch ran the TMA datapath */
   int protocol;                 /* configured: 1 = LL for one-chunk calls, 0 = off */
   int last_ll;                  /* 1 = the most recent call ran the LL kernel */
+  int last_threads;             /* data threads per CTA of the most recent chunked launch */
 } ccube_info_t;
 CCUBE_API ccube_result_t ccube_get_info(ccube_info_t *info);
 

@@ -75,7 +75,8 @@ class Info(ctypes.Structure):
                 ("transport", ctypes.c_int), ("chunk_bytes", ctypes.c_size_t), ("epoch_base", ctypes.c_uint64 * 2),
                 ("last_channels", ctypes.c_int), ("last_ctas", ctypes.c_int),
                 ("datapath", ctypes.c_int), ("last_tma", ctypes.c_int),
-                ("protocol", ctypes.c_int), ("last_ll", ctypes.c_int)]
+                ("protocol", ctypes.c_int), ("last_ll", ctypes.c_int),
+                ("last_threads", ctypes.c_int)]
 
 
 _lib = None

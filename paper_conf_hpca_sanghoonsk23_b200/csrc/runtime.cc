@@ -161,7 +161,7 @@ struct Comm {
   // channels 0 = auto; threads = data threads per CTA: 6 data warps (192) + 2
   // control warps = 256-thread CTAs, 128 registers per thread at two CTAs per SM,
   // 6 vectors per lane and source in flight in the combines (measured)
-  int channels = 0, threads = kDefaultDataThreads, overlap = 1;
+  int channels = 0, threads = 0, overlap = 1;   // threads 0 = auto
   int tree_kind = CCUBE_TREE_SINGLE;
   uint64_t base[kMaxTrees] = {};
   bool have_call = false;
@@ -203,6 +203,7 @@ struct Comm {
   uint32_t ll_epoch = 0;            // LL calls so far (the flag of the next one is +1)
   uint64_t ll_done = 0;             // LL CTAs finished per rank so far
   int last_ll = 0;                  // the most recent call ran the LL kernel
+  int last_threads = 0;             // data threads per CTA of the most recent launch
 };
 
 Comm g;
@@ -651,31 +652,50 @@ ccube_result_t allreduce_impl(void *const *bufs, size_t count, ccube_dtype_t dty
 
   // all CTAs spin on each other: they must be co-resident
   const int nctl = g.split_control ? 2 : 1;
-  const int cta_threads = g.threads + 32 * nctl;  // data warps + the control warp(s)
   // the TMA datapath needs a producer and at least one consumer data warp
   // (AUTO: TMA for the rotated tree set, whose P trees leave few channels and long
   // slices per chunk; the register-staged LSU path for the single and double tree)
   const bool want_tma = g.datapath == CCUBE_DATAPATH_TMA ||
                         (g.datapath == CCUBE_DATAPATH_AUTO && g.ntrees > 2);
-  const int tma = want_tma && g.threads >= 64 ? 1 : 0;
-  auto key = std::make_pair((int)dtype * 2 + (g.sgd ? 1 : 0) + 8 * tma, cta_threads);
-  if (!g.max_blocks.count(key)) {
-    int b = 0;
-    const int rc =
-        query_max_blocks_per_sm(dtype, g.sys_scope, g.sgd, cta_threads, tma, &b);
-    if (rc != cudaSuccess)
-      return fail(CCUBE_ERR_CUDA, "occupancy query failed: %s",
-                  cudaGetErrorString(static_cast<cudaError_t>(rc)));
-    g.max_blocks[key] = b;
-  }
+  // co-resident CTAs per GPU for a CTA of `data` data threads (occupancy, cached)
+  auto capacity = [&](int data, int *cap_out, int *tma_out) -> ccube_result_t {
+    const int tma_ = want_tma && data >= 64 ? 1 : 0;
+    const int cta = data + 32 * nctl;
+    auto key = std::make_pair((int)dtype * 2 + (g.sgd ? 1 : 0) + 8 * tma_, cta);
+    if (!g.max_blocks.count(key)) {
+      int b = 0;
+      const int rc = query_max_blocks_per_sm(dtype, g.sys_scope, g.sgd, cta, tma_, &b);
+      if (rc != cudaSuccess)
+        return fail(CCUBE_ERR_CUDA, "occupancy query failed: %s",
+                    cudaGetErrorString(static_cast<cudaError_t>(rc)));
+      g.max_blocks[key] = b;
+    }
+    *cap_out = g.max_blocks[key] * g.sm_count;
+    *tma_out = tma_;
+    return CCUBE_SUCCESS;
+  };
   // Launch geometry (both ends of an edge must slice chunks alike).
   // J is computed from the maximum task count over ALL processes, so it does not
   // depend on this rank's role in the trees; every setting it depends on is agreed
   // (init's Hello, the collective setters) and every GPU has the same SM count and
   // architecture (init checks it), so every rank computes the same J and the same
   // co-residency verdict without another exchange.
-  const int cap = g.max_blocks[key] * g.sm_count;
   const PlanIn in = plan_in(bytes);
+  int data_threads = g.threads, cap = 0, tma = 0;
+  if (data_threads == 0) {
+    // auto CTA size: 6 data warps with 6 vectors in flight per lane and source (3 KB
+    // blocks) when every channel's slice of a chunk holds >= 3 units of 2 KB, so the
+    // 3 KB blocks tile it; 8 data warps with 2 KB blocks when the slices are short
+    // (many channels: P = 2 / 4), where fewer warps would mean fewer bytes in flight
+    // (round 2).  Deterministic in agreed quantities, like J.
+    CC_TRY(capacity(kDefaultDataThreads, &cap, &tma));
+    const int J0 = g.channels ? g.channels : plan_auto_channels(in, cap);
+    const uint64_t first = bytes < g.chunk_bytes ? bytes : g.chunk_bytes;
+    const uint64_t units = (first + 2047) / 2048;
+    data_threads = units >= 3ull * J0 ? kDefaultDataThreads : 256;
+  }
+  CC_TRY(capacity(data_threads, &cap, &tma));
+  const int cta_threads = data_threads + 32 * nctl;  // data warps + the control warp(s)
   const int J = g.channels ? g.channels : plan_auto_channels(in, cap);
   if (plan_max_tasks(in, J) > cap)
     return fail(CCUBE_ERR_UNSUPPORTED,
@@ -725,6 +745,7 @@ ccube_result_t allreduce_impl(void *const *bufs, size_t count, ccube_dtype_t dty
   g.last_sgd = g.sgd;
   g.last_ctas = tt->n;
   g.last_tma = tma;
+  g.last_threads = data_threads;
   g.last_ll = 0;
   for (int t = 0; t < g.ntrees; ++t) {
     g.last_base[t] = g.base[t];
@@ -1003,9 +1024,10 @@ ccube_result_t ccube_init(const ccube_world_t *world, ccube_tree_kind_t tree_kin
   if (channels < 0 || channels > CCUBE_MAX_CHANNELS)
     return fail(CCUBE_ERR_INVALID_ARG, "CCUBE_CHANNELS %d out of range", channels);
   CC_TRY(check_chunk(chunk_bytes));
-  int threads = env_int("CCUBE_THREADS", kDefaultDataThreads);
-  if (threads < 32 || threads > 256 || threads % 32)
-    return fail(CCUBE_ERR_INVALID_ARG, "CCUBE_THREADS %d out of range [32, 256]", threads);
+  int threads = env_int("CCUBE_THREADS", 0);
+  if (threads != 0 && (threads < 32 || threads > 256 || threads % 32))
+    return fail(CCUBE_ERR_INVALID_ARG, "CCUBE_THREADS %d out of range [32, 256] (0 = auto)",
+                threads);
   const int transport = env_int("CCUBE_TRANSPORT", CCUBE_TRANSPORT_AUTO);
   if (transport < CCUBE_TRANSPORT_AUTO || transport > CCUBE_TRANSPORT_PULL)
     return fail(CCUBE_ERR_INVALID_ARG, "CCUBE_TRANSPORT %d out of range", transport);
@@ -1379,9 +1401,9 @@ ccube_result_t ccube_set_threads(int threads) {
   std::lock_guard<std::mutex> lk(g_mu);
   if (!g.init) return fail(CCUBE_ERR_NOT_INITIALIZED, "ccube_init has not been called");
   const ccube_result_t v =
-      threads < 32 || threads > 256 || threads % 32
-          ? fail(CCUBE_ERR_INVALID_ARG, "threads %d out of range [32, 256] (multiple of 32)",
-                 threads)
+      threads != 0 && (threads < 32 || threads > 256 || threads % 32)
+          ? fail(CCUBE_ERR_INVALID_ARG,
+                 "threads %d out of range [32, 256] (multiple of 32; 0 = auto)", threads)
           : CCUBE_SUCCESS;
   CC_TRY(agree_setting("threads", threads, v));
   g.threads = threads;
@@ -1482,6 +1504,7 @@ ccube_result_t ccube_get_info(ccube_info_t *info) {
   info->last_tma = g.last_tma;
   info->protocol = g.ll;
   info->last_ll = g.last_ll;
+  info->last_threads = g.last_threads;
   return CCUBE_SUCCESS;
 }
 

@@ -229,7 +229,7 @@ def test_multiprocess_settings_are_collective():
     bad = ccube.ERR_INVALID_ARG
     for codes, channels, threads in out:
         assert codes == [bad, 0, bad, bad, 0], codes
-        assert channels == 6 and threads == 192   # the default (rank 1 passed an invalid value)
+        assert channels == 6 and threads == 0   # auto, the default (rank 1 passed an invalid value)
 
 
 def _watchdog(rank, world):

@@ -9,7 +9,11 @@
 # then tools/nvlink_summary.py turns the CSVs into GB/s per rank and launch.
 #
 #   bash tools/nvlink_counters.sh N [extra bench.py args]      (N GPUs on this node)
-# Not a bench number: ncu serialises and instruments the launches.
+# Not a bench number: ncu serialises and instruments the launches.  Needs one GPU per
+# process: on a single shared GPU ncu holds one rank's spinning kernel while the
+# other's waits for it, and the watchdog fires (profiles/r02/l/nvlink_shared.log).
+# bench.py itself reads NVML's NVLink byte counters around its timed region at N > 1
+# (the line's nvlink_counters_rank0), which needs no profiler.
 N=${1:-8}; shift
 OUT=gpurun_out/nvlink_n$N; mkdir -p $OUT
 timeout 1800 ncu --target-processes all --replay-mode application --clock-control none \
