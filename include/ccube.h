@@ -218,9 +218,10 @@ CCUBE_API ccube_result_t ccube_set_threads(int threads);
 #define CCUBE_DATAPATH_TMA 1
 CCUBE_API ccube_result_t ccube_set_datapath(int datapath);
 
-/* Protocol of one-chunk calls (count * elemsize <= chunk_bytes and <= 256 KiB, no
- * fused update): 1 (default; CCUBE_LL env) = the LL ("low latency") kernel — the
- * same tree-0 fold in the same order (bitwise the same result), but every 8 bytes
+/* Protocol of one-chunk calls (count * elemsize <= chunk_bytes and <= the LL
+ * threshold, CCUBE_LL_MAX_BYTES env, default 256 KiB, at most 1 MiB; no fused
+ * update): 1 (default; CCUBE_LL env) = the LL ("low latency") kernel — the same
+ * tree-0 fold in the same order (bitwise the same result), but every 8 bytes
  * of payload travel with the call's epoch and the consumer polls the data itself,
  * so a tree hop costs one store-to-load propagation instead of data stores, a
  * fence, a counter store and a counter poll (eq 3's alpha); the LL lines

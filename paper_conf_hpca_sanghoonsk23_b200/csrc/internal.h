@@ -48,15 +48,17 @@ constexpr size_t kFlagBytes =
 enum BarrierSlot { kBarArrive0 = 0, kBarArrive1 = 1, kBarRelease = 2, kBarSlots = 3 };
 CCUBE_HD inline size_t barrier_offset(int slot) { return kFlagBytes + slot * kFlagStride; }
 
-// Low-latency (LL) protocol for single-chunk messages (<= kLLMaxBytes and <= one
-// chunk): the data carries its own flag.  A 16-byte LL line is {d0, e, d1, e} —
+// Low-latency (LL) protocol for one-chunk messages up to the LL threshold: the data
+// carries its own flag.  A 16-byte LL line is {d0, e, d1, e} —
 // two 4-byte payload words, each paired with the call's epoch e in one 8-byte word
 // (8-byte stores are single-copy atomic), so a reader that sees e twice has the
 // line, with no fence, no counter and no separate flag round trip per hop.
 // Regions per rank, after the barrier counters: the up-lines of child slot 0 and 1
 // (written by the children) and the down-lines (written by the parent), each
 // kLLRegionBytes = 2 x kLLMaxBytes.  Plus one u64 per rank counting finished LL CTAs.
-constexpr size_t kLLMaxBytes = 256u * 1024u;
+constexpr size_t kLLMaxBytes = 1024u * 1024u;   // region capacity; the threshold is
+                                                 // CCUBE_LL_MAX_BYTES (default 256 KiB)
+constexpr size_t kLLDefaultMaxBytes = 256u * 1024u;
 constexpr size_t kLLRegionBytes = 2 * kLLMaxBytes;
 enum LLSlot { kLLUp0 = 0, kLLUp1 = 1, kLLDown = 2, kLLSlots = 3 };
 constexpr size_t kLLBase = kFlagBytes + 4096;   // barrier counters live below

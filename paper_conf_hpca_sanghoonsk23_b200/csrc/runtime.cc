@@ -199,7 +199,8 @@ struct Comm {
   bool use_memop = true;
   bool gate_flush = false;          // memop waits carry CU_STREAM_WAIT_VALUE_FLUSH
   uint64_t bar_epoch = 0;           // ccube_barrier calls so far
-  int ll = 1;                       // CCUBE_LL / ccube_set_protocol: LL for one-chunk calls
+  int ll = 1;                       // CCUBE_LL / ccube_set_protocol: LL for short calls
+  uint64_t ll_max = kLLDefaultMaxBytes;  // CCUBE_LL_MAX_BYTES: the LL threshold
   uint32_t ll_epoch = 0;            // LL calls so far (the flag of the next one is +1)
   uint64_t ll_done = 0;             // LL CTAs finished per rank so far
   int last_ll = 0;                  // the most recent call ran the LL kernel
@@ -561,7 +562,7 @@ ccube_result_t check_chunk(size_t chunk_bytes) {
 // chunk (a3: chunk 0 is on tree 0 for every tree kind), so the result is the chunked
 // path's bit for bit; the epochs of the other trees do not move (K_t = 0).
 ccube_result_t ll_impl(Registration *R, size_t count, ccube_dtype_t dtype, uint64_t E,
-                       void *stream) {
+                       uint64_t K, void *stream) {
   const Tree &tr = g.trees[0];
   LLArgs a;
   memset(&a, 0, sizeof a);
@@ -574,7 +575,7 @@ ccube_result_t ll_impl(Registration *R, size_t count, ccube_dtype_t dtype, uint6
   a.count = count;
   a.epoch = g.ll_epoch + 1;
   a.done_base = g.ll_done;
-  a.enq_value = g.base[0] + 1;
+  a.enq_value = g.base[0] + K;   // every chunk (all on tree 0) has landed
   a.err = g.err_dev;
   a.timeout_ns = g.timeout_ns;
   for (int i = 0; i < g.nlocal; ++i) {
@@ -613,9 +614,9 @@ ccube_result_t ll_impl(Registration *R, size_t count, ccube_dtype_t dtype, uint6
   g.last_ll = 1;
   for (int t = 0; t < g.ntrees; ++t) {
     g.last_base[t] = g.base[t];
-    g.last_K[t] = t == 0 ? 1 : 0;
+    g.last_K[t] = t == 0 ? static_cast<uint32_t>(K) : 0;
   }
-  g.base[0] += 1;
+  g.base[0] += K;
   return CCUBE_SUCCESS;
 }
 
@@ -647,7 +648,11 @@ ccube_result_t allreduce_impl(void *const *bufs, size_t count, ccube_dtype_t dty
 
   const uint64_t E = g.chunk_bytes / es;
   const uint64_t K = (count + E - 1) / E;
-  if (g.ll && !g.sgd && K == 1 && bytes <= kLLMaxBytes) return ll_impl(R, count, dtype, E, stream);
+  // one-chunk messages up to the LL threshold: the LL protocol — the same tree-0 fold,
+  // one kernel without counters or fences.  (Multi-chunk single-tree messages on LL
+  // measured no faster than the chunked kernel from 512 KiB up: DESIGN §10.)
+  if (g.ll && !g.sgd && K == 1 && bytes <= g.ll_max)
+    return ll_impl(R, count, dtype, E, K, stream);
   if (K > 0xffffffffull) return fail(CCUBE_ERR_INVALID_ARG, "too many chunks");
 
   // all CTAs spin on each other: they must be co-resident
@@ -844,6 +849,7 @@ struct Hello {
   // the launch geometry is computed locally from the occupancy: every GPU must be
   // the same architecture with the same SM count
   int32_t sm_count, cc_major, cc_minor, ll;
+  uint64_t ll_max;
   uint64_t chunk_bytes;
   char busid[32];
   int8_t place[CCUBE_MAX_RANKS];  // the placement (R19), identity when none was set
@@ -1054,6 +1060,10 @@ ccube_result_t ccube_init(const ccube_world_t *world, ccube_tree_kind_t tree_kin
   g.backoff_ns = env_int("CCUBE_BACKOFF_NS", 64);
   g.debug_nodep = env_int("CCUBE_DEBUG_NODEP", 0);
   g.ll = env_int("CCUBE_LL", 1) != 0 ? 1 : 0;
+  {
+    const int m = env_int("CCUBE_LL_MAX_BYTES", static_cast<int>(kLLDefaultMaxBytes));
+    g.ll_max = m < 0 ? 0 : (static_cast<uint64_t>(m) > kLLMaxBytes ? kLLMaxBytes : m);
+  }
   g.datapath = env_int("CCUBE_DATAPATH", CCUBE_DATAPATH_AUTO);
   if (g.datapath != CCUBE_DATAPATH_LSU && g.datapath != CCUBE_DATAPATH_TMA)
     g.datapath = CCUBE_DATAPATH_AUTO;
@@ -1082,6 +1092,7 @@ ccube_result_t ccube_init(const ccube_world_t *world, ccube_tree_kind_t tree_kin
   mine.l2_hints = g.l2_hints;
   mine.split_control = g.split_control;
   mine.ll = g.ll;
+  mine.ll_max = g.ll_max;
   if (cudaDeviceGetAttribute(&mine.sm_count, cudaDevAttrMultiProcessorCount, g.device) !=
           cudaSuccess ||
       cudaDeviceGetAttribute(&mine.cc_major, cudaDevAttrComputeCapabilityMajor, g.device) !=
@@ -1124,7 +1135,7 @@ ccube_result_t ccube_init(const ccube_world_t *world, ccube_tree_kind_t tree_kin
     if (h.channels != mine.channels || h.threads != mine.threads ||
         h.datapath != mine.datapath || h.transport != mine.transport ||
         h.l2_hints != mine.l2_hints || h.split_control != mine.split_control ||
-        h.ll != mine.ll) {
+        h.ll != mine.ll || h.ll_max != mine.ll_max) {
       g = Comm();
       return fail(CCUBE_ERR_INVALID_ARG,
                   "ranks disagree on the launch settings (process %d: CCUBE_CHANNELS %d "

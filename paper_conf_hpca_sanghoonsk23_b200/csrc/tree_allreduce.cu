@@ -1156,19 +1156,32 @@ __device__ __forceinline__ void ll_store(char *p, uint32_t d0, uint32_t d1, uint
                  "r"(d1), "r"(e) : "memory");
 }
 
-// Poll an LL line until both of its 8-byte words carry the epoch.
+// Poll the LL lines l0, l0 + stride, ... (kLLBatch of them, those < lines) until each
+// carries the epoch; the loads of the lines still missing are issued together.
+constexpr int kLLBatch = 4;
 template <bool SYS>
-__device__ __forceinline__ bool ll_wait(const char *p, uint32_t e, const LLArgs &a, uint64_t &t0,
-                                        uint32_t &d0, uint32_t &d1) {
+__device__ __forceinline__ bool ll_wait_batch(const char *base, uint64_t l0, uint64_t stride,
+                                              uint64_t lines, uint32_t e, const LLArgs &a,
+                                              uint64_t &t0, uint32_t (&d0)[kLLBatch],
+                                              uint32_t (&d1)[kLLBatch]) {
+  uint32_t missing = 0;
+#pragma unroll
+  for (int i = 0; i < kLLBatch; ++i)
+    if (l0 + i * stride < lines) missing |= 1u << i;
   uint32_t spins = 0;
-  for (;;) {
-    const uint4 v = ll_load<SYS>(p);
-    if (v.y == e && v.w == e) {
-      d0 = v.x;
-      d1 = v.z;
-      return true;
-    }
-    if ((++spins & 255) == 0) {
+  while (missing) {
+    uint4 v[kLLBatch];
+#pragma unroll
+    for (int i = 0; i < kLLBatch; ++i)
+      if (missing & (1u << i)) v[i] = ll_load<SYS>(base + 16 * (l0 + i * stride));
+#pragma unroll
+    for (int i = 0; i < kLLBatch; ++i)
+      if ((missing & (1u << i)) && v[i].y == e && v[i].w == e) {
+        d0[i] = v[i].x;
+        d1[i] = v[i].z;
+        missing &= ~(1u << i);
+      }
+    if (missing && (++spins & 255) == 0) {
       const uint64_t now = globaltimer();
       if (t0 == 0) t0 = now;
       if (*reinterpret_cast<volatile int *>(a.err) != 0) return false;
@@ -1176,7 +1189,7 @@ __device__ __forceinline__ bool ll_wait(const char *p, uint32_t e, const LLArgs 
         volatile int *err = reinterpret_cast<volatile int *>(a.err);
         err[1] = static_cast<int>(blockIdx.x);
         err[2] = static_cast<int>(e);
-        err[3] = static_cast<int>(v.y);
+        err[3] = static_cast<int>(missing);
         __threadfence_system();
         err[0] = 4;  // 4 = LL watchdog
         __threadfence_system();
@@ -1184,26 +1197,28 @@ __device__ __forceinline__ bool ll_wait(const char *p, uint32_t e, const LLArgs 
       }
     }
   }
+  return true;
 }
 
 // One node's combine on a word pair: own, then each child's partial in ascending
 // rank, left to right (R2); bf16 accumulates both halves in fp32 and rounds once
 // per node output (R3); a leaf's own bits are forwarded untouched.
 template <int DT>
-__device__ __forceinline__ uint32_t ll_combine(uint32_t own, const uint32_t *c, int n) {
+__device__ __forceinline__ uint32_t ll_combine(uint32_t own, uint32_t c0, uint32_t c1, int n) {
   if (n == 0) return own;
   if (DT == kInt32) {
-    for (int i = 0; i < n; ++i) own += c[i];
+    own += c0;
+    if (n > 1) own += c1;
     return own;
   } else if (DT == kFloat32) {
-    float f = __uint_as_float(own);
-    for (int i = 0; i < n; ++i) f = __fadd_rn(f, __uint_as_float(c[i]));
+    float f = __fadd_rn(__uint_as_float(own), __uint_as_float(c0));
+    if (n > 1) f = __fadd_rn(f, __uint_as_float(c1));
     return __float_as_uint(f);
   } else {
-    float lo = bf_lo(own), hi = bf_hi(own);
-    for (int i = 0; i < n; ++i) {
-      lo = __fadd_rn(lo, bf_lo(c[i]));
-      hi = __fadd_rn(hi, bf_hi(c[i]));
+    float lo = __fadd_rn(bf_lo(own), bf_lo(c0)), hi = __fadd_rn(bf_hi(own), bf_hi(c0));
+    if (n > 1) {
+      lo = __fadd_rn(lo, bf_lo(c1));
+      hi = __fadd_rn(hi, bf_hi(c1));
     }
     return bf_round(lo) | (bf_round(hi) << 16);
   }
@@ -1236,34 +1251,54 @@ __global__ void __launch_bounds__(512) ll_kernel(const LLArgs a) {
   const uint32_t e = a.epoch;
   uint64_t t0 = 0;
   bool ok = true;
+  // Each thread takes kLLBatch lines (l0, l0 + stride, ...) at a time, so its loads
+  // and polls of those lines are in flight together.
   // phase 1: reduce-up (and the root's turnaround)
-  for (uint64_t l = static_cast<uint64_t>(part) * blockDim.x + threadIdx.x; l < lines && ok;
-       l += stride) {
-    uint32_t w0 = ll_get(me.buf, 2 * l, nbytes), w1 = ll_get(me.buf, 2 * l + 1, nbytes);
-    uint32_t c0[kMaxChildren], c1[kMaxChildren];
-    for (int s = 0; s < me.nchild && ok; ++s)
-      ok = ll_wait<SYS>(me.up_in[s] + 16 * l, e, a, t0, c0[s], c1[s]);
+  for (uint64_t l0 = static_cast<uint64_t>(part) * blockDim.x + threadIdx.x; l0 < lines && ok;
+       l0 += stride * kLLBatch) {
+    uint32_t w0[kLLBatch], w1[kLLBatch], c0[kMaxChildren][kLLBatch] = {}, c1[kMaxChildren][kLLBatch] = {};
+#pragma unroll
+    for (int i = 0; i < kLLBatch; ++i) {
+      const uint64_t l = l0 + i * stride;
+      w0[i] = l < lines ? ll_get(me.buf, 2 * l, nbytes) : 0;
+      w1[i] = l < lines ? ll_get(me.buf, 2 * l + 1, nbytes) : 0;
+    }
+#pragma unroll
+    for (int s = 0; s < kMaxChildren; ++s)
+      if (s < me.nchild && ok)
+        ok = ll_wait_batch<SYS>(me.up_in[s], l0, stride, lines, e, a, t0, c0[s], c1[s]);
     if (!ok) break;
-    w0 = ll_combine<DT>(w0, c0, me.nchild);
-    w1 = ll_combine<DT>(w1, c1, me.nchild);
-    if (me.up_out) {
-      ll_store<SYS>(me.up_out + 16 * l, w0, w1, e);
-    } else {  // root: final
-      ll_put(me.buf, 2 * l, nbytes, w0);
-      ll_put(me.buf, 2 * l + 1, nbytes, w1);
-      for (int s = 0; s < me.nchild; ++s) ll_store<SYS>(me.down_out[s] + 16 * l, w0, w1, e);
+#pragma unroll
+    for (int i = 0; i < kLLBatch; ++i) {
+      const uint64_t l = l0 + i * stride;
+      if (l >= lines) break;
+      const uint32_t r0 = ll_combine<DT>(w0[i], c0[0][i], c0[1][i], me.nchild);
+      const uint32_t r1 = ll_combine<DT>(w1[i], c1[0][i], c1[1][i], me.nchild);
+      if (me.up_out) {
+        ll_store<SYS>(me.up_out + 16 * l, r0, r1, e);
+      } else {  // root: final
+        ll_put(me.buf, 2 * l, nbytes, r0);
+        ll_put(me.buf, 2 * l + 1, nbytes, r1);
+        for (int s = 0; s < me.nchild; ++s) ll_store<SYS>(me.down_out[s] + 16 * l, r0, r1, e);
+      }
     }
   }
   // phase 2: broadcast-down
   if (me.up_out) {
-    for (uint64_t l = static_cast<uint64_t>(part) * blockDim.x + threadIdx.x; l < lines && ok;
-         l += stride) {
-      uint32_t w0, w1;
-      ok = ll_wait<SYS>(me.down_in + 16 * l, e, a, t0, w0, w1);
+    for (uint64_t l0 = static_cast<uint64_t>(part) * blockDim.x + threadIdx.x;
+         l0 < lines && ok; l0 += stride * kLLBatch) {
+      uint32_t w0[kLLBatch], w1[kLLBatch];
+      ok = ll_wait_batch<SYS>(me.down_in, l0, stride, lines, e, a, t0, w0, w1);
       if (!ok) break;
-      ll_put(me.buf, 2 * l, nbytes, w0);
-      ll_put(me.buf, 2 * l + 1, nbytes, w1);
-      for (int s = 0; s < me.nchild; ++s) ll_store<SYS>(me.down_out[s] + 16 * l, w0, w1, e);
+#pragma unroll
+      for (int i = 0; i < kLLBatch; ++i) {
+        const uint64_t l = l0 + i * stride;
+        if (l >= lines) break;
+        ll_put(me.buf, 2 * l, nbytes, w0[i]);
+        ll_put(me.buf, 2 * l + 1, nbytes, w1[i]);
+        for (int s = 0; s < me.nchild; ++s)
+          ll_store<SYS>(me.down_out[s] + 16 * l, w0[i], w1[i], e);
+      }
     }
   }
   // the rank's last CTA to finish publishes the Enqueue Semaphore: every final word
