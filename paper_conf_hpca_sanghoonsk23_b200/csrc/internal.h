@@ -34,7 +34,11 @@ constexpr int kMaxChildren = 2;
 constexpr int kFlagStride = 64;  // bytes between two counters
 constexpr int kFlagStrideU64 = kFlagStride / 8;
 
-enum FlagKind { kUpHead0 = 0, kUpHead1 = 1, kEnq = 2, kUpd = 3, kNumFlagKinds = 4 };
+// kHalf0/1: progress of the two CTAs of a split task (see Task::halves), written by
+// each half for the other.
+enum FlagKind {
+  kUpHead0 = 0, kUpHead1 = 1, kEnq = 2, kUpd = 3, kHalf0 = 4, kHalf1 = 5, kNumFlagKinds = 6
+};
 
 CCUBE_HD inline size_t flag_offset(int tree, int kind, int ch) {
   return ((static_cast<size_t>(tree) * kNumFlagKinds + kind) * kMaxChannels + ch) * kFlagStride;
@@ -97,6 +101,7 @@ struct TreeParams {
   int child_interior[kMaxChildren]; // child has children: its buffer is re-read (DOWN)
   char *w;                          // own fp32 weights (fused SGD, f2), same layout as buf
   uint64_t *upd;                    // own "weights updated" counter (channel 0)
+  uint64_t *half_slot[2];           // own progress slots of a split task's halves (channel 0)
 };
 
 // UPDATE: a leaf's fused-SGD task (f2) — waits for its chunks to land, then
@@ -105,11 +110,18 @@ enum Role { kRoleUp = 0, kRoleDown = 1, kRoleUpdate = 2 };
 
 enum { kAllChannels = -1 };  // a pulled leaf's single task covers every channel
 
+// A task normally runs on one CTA.  With CCUBE_SPLIT_HEADS=1 the pipeline's head — an
+// UP task whose children are all pulled leaves, which reads 3 of the DRAM input
+// streams — is split over two CTAs (halves = 2): half h's data warps take every other
+// block of the channel's slices, and the channel's counters are published (monotone
+// max) once BOTH halves are past a chunk.  Off by default (measured slower).
 struct Task {
   int16_t local_rank;
   int16_t tree;
   int16_t role;
   int16_t channel;   // kAllChannels for a pulled leaf
+  int16_t half;      // 0, or 1 for the second CTA of a split task
+  int16_t halves;    // 1, or 2 for a split task
 };
 
 struct LaunchArgs {

@@ -11,6 +11,15 @@ bool plan_edge_is_pull(int transport, int nlocal, int child, int parent) {
   return child / nlocal == parent / nlocal;
 }
 
+bool plan_is_head(const PlanIn &in, const Tree &tr, int r) {
+  if (tr.nchild[r] == 0) return false;
+  for (int s = 0; s < tr.nchild[r]; ++s) {
+    const int c = tr.child[r][s];
+    if (tr.nchild[c] != 0 || !plan_edge_is_pull(in.transport, in.nlocal, c, r)) return false;
+  }
+  return true;
+}
+
 int plan_tasks_of_proc(const PlanIn &in, int proc, int J) {
   int n = 0;
   for (int i = 0; i < in.nlocal; ++i) {
@@ -24,7 +33,7 @@ int plan_tasks_of_proc(const PlanIn &in, int proc, int J) {
         n += 1;  // a pulled leaf: one CTA publishes every channel
         continue;
       }
-      n += J;                                                  // UP
+      n += (in.split_heads && plan_is_head(in, tr, r)) ? 2 * J : J;  // UP
       if (tr.nchild[r] > 0 && (!root || !in.overlap)) n += J;  // DOWN
     }
   }

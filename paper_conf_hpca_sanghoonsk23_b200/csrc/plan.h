@@ -25,7 +25,13 @@ struct PlanIn {
   bool sgd;            // fused SGD update (adds an UPDATE task per leaf and channel)
   uint64_t bytes;      // buffer bytes of this call
   uint64_t chunk_bytes;
+  bool split_heads;    // the pipeline's head tasks run on two CTAs per channel
 };
+
+// The pipeline's head: an UP task whose children are all pulled leaves (it reads its
+// own and its children's inputs from DRAM).  Split over two CTAs per channel when
+// PlanIn::split_heads.
+bool plan_is_head(const PlanIn &in, const Tree &tr, int r);
 
 // Edge child -> parent: PULL (the parent reads the child's partial in place) when
 // both ranks live in the same process (same GPU) under AUTO; PUSH otherwise.

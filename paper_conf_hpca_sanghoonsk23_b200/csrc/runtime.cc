@@ -199,6 +199,7 @@ struct Comm {
   bool use_memop = true;
   bool gate_flush = false;          // memop waits carry CU_STREAM_WAIT_VALUE_FLUSH
   uint64_t bar_epoch = 0;           // ccube_barrier calls so far
+  int split_heads = 0;              // CCUBE_SPLIT_HEADS: the pipeline's head on 2 CTAs/channel
   int ll = 1;                       // CCUBE_LL / ccube_set_protocol: LL for short calls
   uint64_t ll_max = kLLDefaultMaxBytes;  // CCUBE_LL_MAX_BYTES: the LL threshold
   uint32_t ll_epoch = 0;            // LL calls so far (the flag of the next one is +1)
@@ -303,8 +304,19 @@ bool edge_is_pull(int child, int parent) {
   return plan_edge_is_pull(g.transport, g.nlocal, child, parent);
 }
 
+// The TMA datapath is chosen by the datapath setting and the tree kind (AUTO: TMA
+// for the rotated set); the split of the pipeline's head tasks runs on the LSU path
+// with the two control warps, without the fused update.
+bool want_tma() {
+  return g.datapath == CCUBE_DATAPATH_TMA || (g.datapath == CCUBE_DATAPATH_AUTO && g.ntrees > 2);
+}
+bool split_heads_now() {
+  return g.split_heads && !g.sgd && !want_tma() && g.split_control;
+}
+
 PlanIn plan_in(uint64_t bytes) {
   PlanIn in;
+  in.split_heads = split_heads_now();
   in.trees = g.trees;
   in.ntrees = g.ntrees;
   in.world = g.world;
@@ -375,6 +387,8 @@ ccube_result_t build_params(Registration *R) {
       }
       p.enq = reinterpret_cast<uint64_t *>(fl + flag_offset(t, kEnq, 0));
       p.upd = reinterpret_cast<uint64_t *>(fl + flag_offset(t, kUpd, 0));
+      for (int h = 0; h < 2; ++h)
+        p.half_slot[h] = reinterpret_cast<uint64_t *>(fl + flag_offset(t, kHalf0 + h, 0));
       p.w = g.sgd ? g.sgd_w[i] : nullptr;
       const int par = tr.parent[r];
       if (par < 0) {
@@ -512,12 +526,18 @@ void order_tasks(std::vector<Task> &ts) {
 }
 
 ccube_result_t get_tasks(int channels, int overlap, TaskTable **out) {
-  auto key = std::make_pair(channels, overlap * 2 + (g.sgd ? 1 : 0));
+  const bool split = split_heads_now();
+  auto key = std::make_pair(channels, overlap * 2 + (g.sgd ? 1 : 0) + (split ? 4 : 0));
   auto it = g.tasks.find(key);
   if (it != g.tasks.end()) {
     *out = &it->second;
     return CCUBE_SUCCESS;
   }
+  const PlanIn in = plan_in(0);
+  auto task = [](int i, int t, int role, int j, int half = 0, int halves = 1) {
+    return Task{(int16_t)i, (int16_t)t, (int16_t)role, (int16_t)j, (int16_t)half,
+                (int16_t)halves};
+  };
   std::vector<Task> ts;
   for (int i = 0; i < g.nlocal; ++i) {
     const int r = g.rank0 + i;
@@ -525,18 +545,19 @@ ccube_result_t get_tasks(int channels, int overlap, TaskTable **out) {
       const Tree &tr = g.trees[t];
       const bool root = tr.parent[r] < 0;
       if (!root && tr.nchild[r] == 0 && g.sgd)  // a leaf's fused SGD step (f2)
-        for (int j = 0; j < channels; ++j)
-          ts.push_back(Task{(int16_t)i, (int16_t)t, (int16_t)kRoleUpdate, (int16_t)j});
+        for (int j = 0; j < channels; ++j) ts.push_back(task(i, t, kRoleUpdate, j));
       if (!root && tr.nchild[r] == 0 && edge_is_pull(r, tr.parent[r])) {
-        ts.push_back(Task{(int16_t)i, (int16_t)t, (int16_t)kRoleUp, (int16_t)kAllChannels});
+        ts.push_back(task(i, t, kRoleUp, kAllChannels));
         continue;
       }
       const bool down = tr.nchild[r] > 0 && (!root || !overlap);
-      for (int j = 0; j < channels; ++j)
-        ts.push_back(Task{(int16_t)i, (int16_t)t, (int16_t)kRoleUp, (int16_t)j});
+      const bool head = split && plan_is_head(in, tr, r);
+      for (int j = 0; j < channels; ++j) {
+        ts.push_back(task(i, t, kRoleUp, j, 0, head ? 2 : 1));
+        if (head) ts.push_back(task(i, t, kRoleUp, j, 1, 2));
+      }
       if (down)
-        for (int j = 0; j < channels; ++j)
-          ts.push_back(Task{(int16_t)i, (int16_t)t, (int16_t)kRoleDown, (int16_t)j});
+        for (int j = 0; j < channels; ++j) ts.push_back(task(i, t, kRoleDown, j));
     }
   }
   order_tasks(ts);
@@ -660,11 +681,10 @@ ccube_result_t allreduce_impl(void *const *bufs, size_t count, ccube_dtype_t dty
   // the TMA datapath needs a producer and at least one consumer data warp
   // (AUTO: TMA for the rotated tree set, whose P trees leave few channels and long
   // slices per chunk; the register-staged LSU path for the single and double tree)
-  const bool want_tma = g.datapath == CCUBE_DATAPATH_TMA ||
-                        (g.datapath == CCUBE_DATAPATH_AUTO && g.ntrees > 2);
+  const bool tma_wanted = want_tma();
   // co-resident CTAs per GPU for a CTA of `data` data threads (occupancy, cached)
   auto capacity = [&](int data, int *cap_out, int *tma_out) -> ccube_result_t {
-    const int tma_ = want_tma && data >= 64 ? 1 : 0;
+    const int tma_ = tma_wanted && data >= 64 ? 1 : 0;
     const int cta = data + 32 * nctl;
     auto key = std::make_pair((int)dtype * 2 + (g.sgd ? 1 : 0) + 8 * tma_, cta);
     if (!g.max_blocks.count(key)) {
@@ -850,6 +870,7 @@ struct Hello {
   // the same architecture with the same SM count
   int32_t sm_count, cc_major, cc_minor, ll;
   uint64_t ll_max;
+  int32_t split_heads, pad2;
   uint64_t chunk_bytes;
   char busid[32];
   int8_t place[CCUBE_MAX_RANKS];  // the placement (R19), identity when none was set
@@ -1060,6 +1081,9 @@ ccube_result_t ccube_init(const ccube_world_t *world, ccube_tree_kind_t tree_kin
   g.backoff_ns = env_int("CCUBE_BACKOFF_NS", 64);
   g.debug_nodep = env_int("CCUBE_DEBUG_NODEP", 0);
   g.ll = env_int("CCUBE_LL", 1) != 0 ? 1 : 0;
+  // off by default: measured slower (round 2) — the head then outruns the
+  // stages after it, which lose CTAs and the L2 residency of the head's partials
+  g.split_heads = env_int("CCUBE_SPLIT_HEADS", 0) != 0 ? 1 : 0;
   {
     const int m = env_int("CCUBE_LL_MAX_BYTES", static_cast<int>(kLLDefaultMaxBytes));
     g.ll_max = m < 0 ? 0 : (static_cast<uint64_t>(m) > kLLMaxBytes ? kLLMaxBytes : m);
@@ -1093,6 +1117,7 @@ ccube_result_t ccube_init(const ccube_world_t *world, ccube_tree_kind_t tree_kin
   mine.split_control = g.split_control;
   mine.ll = g.ll;
   mine.ll_max = g.ll_max;
+  mine.split_heads = g.split_heads;
   if (cudaDeviceGetAttribute(&mine.sm_count, cudaDevAttrMultiProcessorCount, g.device) !=
           cudaSuccess ||
       cudaDeviceGetAttribute(&mine.cc_major, cudaDevAttrComputeCapabilityMajor, g.device) !=
@@ -1135,12 +1160,13 @@ ccube_result_t ccube_init(const ccube_world_t *world, ccube_tree_kind_t tree_kin
     if (h.channels != mine.channels || h.threads != mine.threads ||
         h.datapath != mine.datapath || h.transport != mine.transport ||
         h.l2_hints != mine.l2_hints || h.split_control != mine.split_control ||
-        h.ll != mine.ll || h.ll_max != mine.ll_max) {
+        h.ll != mine.ll || h.ll_max != mine.ll_max || h.split_heads != mine.split_heads) {
       g = Comm();
       return fail(CCUBE_ERR_INVALID_ARG,
                   "ranks disagree on the launch settings (process %d: CCUBE_CHANNELS %d "
                   "CCUBE_THREADS %d CCUBE_DATAPATH %d CCUBE_TRANSPORT %d CCUBE_L2_HINTS %d "
-                  "CCUBE_SPLIT_CONTROL %d, or CCUBE_LL; here %d %d %d %d %d %d)",
+                  "CCUBE_SPLIT_CONTROL %d, or CCUBE_LL[_MAX_BYTES] / CCUBE_SPLIT_HEADS; here "
+                  "%d %d %d %d %d %d)",
                   p, h.channels, h.threads, h.datapath, h.transport, h.l2_hints,
                   h.split_control, mine.channels, mine.threads, mine.datapath, mine.transport,
                   mine.l2_hints, mine.split_control);
@@ -1320,6 +1346,7 @@ ccube_result_t ccube_plan_launch(int P, ccube_tree_kind_t kind, int nlocal, int 
   in.sgd = false;
   in.bytes = bytes;
   in.chunk_bytes = chunk_bytes;
+  in.split_heads = false;   // the default (CCUBE_SPLIT_HEADS=0)
   const int J = channels ? channels : plan_auto_channels(in, cap_ctas);
   *channels_out = J;
   *ctas_out = plan_tasks_of_proc(in, rank / nlocal, J);

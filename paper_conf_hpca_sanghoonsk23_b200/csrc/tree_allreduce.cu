@@ -518,6 +518,69 @@ __device__ __forceinline__ void publish(const LaunchArgs &a, const TreeParams &p
   }
 }
 
+// A split task's release of chunks [pub, d): as publish(), but several writers (the
+// two halves) may store each counter, so every store is a monotone max with release
+// semantics (`red.release.max`): a half that publishes an older minimum can never move
+// a counter back.
+template <bool SYS>
+__device__ __forceinline__ void red_max_release(uint64_t *p, uint64_t v) {
+  if (SYS)
+    asm volatile("red.release.sys.global.max.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+  else
+    asm volatile("red.release.gpu.global.max.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+template <bool SYS>
+__device__ __forceinline__ void fence_sc() {
+  if (SYS)
+    asm volatile("fence.sc.sys;" ::: "memory");
+  else
+    asm volatile("fence.sc.gpu;" ::: "memory");
+}
+
+template <bool SYS>
+__device__ __forceinline__ void publish_max(const LaunchArgs &a, const TreeParams &p, int role,
+                                            int t, int j, uint32_t pub, uint32_t d,
+                                            uint64_t base) {
+  const int stride = j * kFlagStrideU64;
+  const uint64_t v = base + d;
+  if (role == kRoleUp && !p.is_root) {
+    red_max_release<SYS>(p.head_out + stride, v);
+    if (a.trace_up) trace_landing(a, p.self_local, t, pub, d, j, a.trace_up);
+    return;
+  }
+  if (role == kRoleUp) {  // root: the chunk is final in my own buffer
+    red_max_release<SYS>(p.enq + stride, v);
+    trace_landing(a, p.self_local, t, pub, d, j);
+    if (!a.overlap) return;
+  }
+  for (int s = 0; s < p.nchild; ++s) {
+    red_max_release<SYS>(p.child_enq[s] + stride, v);
+    trace_landing(a, p.child_local[s], t, pub, d, j);
+  }
+}
+
+// Half h of a split task has finished chunks < d (its own warps).  It records that
+// in its progress slot, reads the other half's, and releases downstream the minimum
+// of the two if that advanced.  The store-then-load on two slots is separated by a
+// sequentially consistent fence in both halves, so of two halves finishing the same
+// chunk at least one sees the other's progress: the minimum always gets published.
+template <bool SYS>
+__device__ __forceinline__ uint32_t publish_half(const LaunchArgs &a, const TreeParams &p,
+                                                 int role, int t, int j, int half, uint32_t d,
+                                                 uint32_t published, uint64_t base) {
+  const int stride = j * kFlagStrideU64;
+  fence_release<SYS>();                                 // my warps' stores, then my slot
+  st_relaxed<SYS>(p.half_slot[half] + stride, base + d);
+  fence_sc<SYS>();
+  const uint64_t o = ld_acquire<SYS>(p.half_slot[half ^ 1] + stride);
+  uint32_t m = o > base ? static_cast<uint32_t>(o - base < d ? o - base : d) : 0;
+  if (m > published) {
+    publish_max<SYS>(a, p, role, t, j, published, m, base);
+    return m;
+  }
+  return published;
+}
+
 // Leaf completion: the kernel completes only once the whole result has landed.
 template <bool SYS>
 __device__ __forceinline__ void leaf_wait(const LaunchArgs &a, const TreeParams &p, int role,
@@ -688,12 +751,13 @@ __device__ void poll_warp(const LaunchArgs &a, const TreeParams &p, int role, in
 
 template <bool SYS>
 __device__ void publish_warp(const LaunchArgs &a, const TreeParams &p, int role, int t, int j,
-                             int W, Shared &sh) {
+                             int W, Shared &sh, int half, int halves) {
   const int lane = threadIdx.x & 31;
   const uint32_t K = a.K[t];
   const uint64_t base = a.base[t];
   const int stride = j * kFlagStrideU64;
-  uint32_t pub = 0;
+  uint32_t pub = 0;        // chunks my own warps finished
+  uint32_t published = 0;  // split task: chunks released downstream (lane 0's view)
   Watch wd;
   watch_reset(wd);
   while (pub < K) {
@@ -701,10 +765,16 @@ __device__ void publish_warp(const LaunchArgs &a, const TreeParams &p, int role,
     d = warp_min(d);
     if (d > pub) {
       __syncwarp();
-      if (lane == 0) publish<SYS>(a, p, role, t, j, pub, static_cast<uint32_t>(d), base);
+      if (lane == 0) {
+        if (halves == 1)
+          publish<SYS>(a, p, role, t, j, pub, static_cast<uint32_t>(d), base);
+        else
+          published = publish_half<SYS>(a, p, role, t, j, half, static_cast<uint32_t>(d),
+                                        published, base);
+      }
       pub = static_cast<uint32_t>(d);
       watch_reset(wd);
-    } else {
+    } else {  // (a split task needs no retry: the half that is behind publishes)
       if (*reinterpret_cast<volatile int *>(&sh.abort)) return;
       if (!watch_tick(wd, a, base + pub + 1, base + pub)) {
         if (lane == 0) {
@@ -737,7 +807,7 @@ __device__ __forceinline__ uint4 sgd4(const uint4 &w, const uint4 &g, float alph
 
 template <int DT, int NIN, int NOUT, int U, bool SGD>
 __device__ void lsu_stream(const LaunchArgs &a, const Endpoints &e, int t, int j, int w, int W,
-                           Shared &sh) {
+                           Shared &sh, int iw, int iW) {
   constexpr int ES = DT == kBFloat16 ? 2 : 4;
   constexpr uint32_t kSeg = 512u * U;
   const int lane = threadIdx.x & 31;
@@ -749,7 +819,7 @@ __device__ void lsu_stream(const LaunchArgs &a, const Endpoints &e, int t, int j
   uint64_t dpol[NOUT > 0 ? NOUT : 1];
 #pragma unroll
   for (int q = 0; q < NOUT; ++q) dpol[q] = (e.keep >> q) & 1u ? pol.last : pol.first;
-  BlockIter it = iter_begin<kSeg>(g, w);
+  BlockIter it = iter_begin<kSeg>(g, iw);  // iw / iW: this warp among the task's CTAs
   while (it.k < g.K) {
     const uint32_t k = it.k;
     if (k >= ready) {
@@ -778,7 +848,7 @@ __device__ void lsu_stream(const LaunchArgs &a, const Endpoints &e, int t, int j
         if constexpr (SGD) wv[u] = ld_hint(e.w + off + lane * 16 + 512u * u, pol.first);
       }
     }
-    it.s += W;  // advance while the loads are in flight (the loop is latency bound)
+    it.s += iW;  // advance while the loads are in flight (the loop is latency bound)
     iter_settle<kSeg>(g, it);
 #pragma unroll
     for (int u = 0; u < U; ++u) {
@@ -816,22 +886,22 @@ __device__ void lsu_stream(const LaunchArgs &a, const Endpoints &e, int t, int j
 
 template <int DT, int NIN, bool SGD, int MAXT>
 __device__ __forceinline__ void lsu_nout(const LaunchArgs &a, const Endpoints &e, int t, int j,
-                                         int w, int W, Shared &sh) {
+                                         int w, int W, Shared &sh, int iw, int iW) {
   // block = 2 KB (copies and combines); build-time overrides for experiments
   constexpr int U = NIN == 1 ? (MAXT <= 256 ? CCUBE_U_COPY_S : CCUBE_U_COPY) : u_combine(MAXT);
   if constexpr (SGD && DT == kFloat32 && NIN <= 2) {
     if (e.sgd) {  // root UP (NIN 2), interior DOWN and leaf UPDATE (NIN 1); U = 4 (2 KB)
       switch (e.nout) {
-        case 0: lsu_stream<DT, NIN, 0, 4, true>(a, e, t, j, w, W, sh); return;
-        case 1: lsu_stream<DT, NIN, 1, 4, true>(a, e, t, j, w, W, sh); return;
-        default: lsu_stream<DT, NIN, 2, 4, true>(a, e, t, j, w, W, sh); return;
+        case 0: lsu_stream<DT, NIN, 0, 4, true>(a, e, t, j, w, W, sh, iw, iW); return;
+        case 1: lsu_stream<DT, NIN, 1, 4, true>(a, e, t, j, w, W, sh, iw, iW); return;
+        default: lsu_stream<DT, NIN, 2, 4, true>(a, e, t, j, w, W, sh, iw, iW); return;
       }
     }
   }
   switch (e.nout) {
-    case 1: lsu_stream<DT, NIN, 1, U, false>(a, e, t, j, w, W, sh); break;
-    case 2: lsu_stream<DT, NIN, 2, U, false>(a, e, t, j, w, W, sh); break;
-    default: lsu_stream<DT, NIN, 3, U, false>(a, e, t, j, w, W, sh); break;
+    case 1: lsu_stream<DT, NIN, 1, U, false>(a, e, t, j, w, W, sh, iw, iW); break;
+    case 2: lsu_stream<DT, NIN, 2, U, false>(a, e, t, j, w, W, sh, iw, iW); break;
+    default: lsu_stream<DT, NIN, 3, U, false>(a, e, t, j, w, W, sh, iw, iW); break;
   }
 }
 
@@ -1041,7 +1111,8 @@ __device__ void tma_data_warp(const LaunchArgs &a, const TreeParams &p, int role
 
 template <int DT, bool SGD, int MAXT>
 __device__ void data_warp(const LaunchArgs &a, const TreeParams &p, int role, int t, int j,
-                          int w, int W, Shared &sh) {
+                          int w, int W, Shared &sh, int half, int halves) {
+  const int iw = half * W + w, iW = halves * W;  // a split task's halves interleave blocks
   Endpoints e = endpoints(a, p, role);
   if (!SGD) e.sgd = false;
   if (e.nout == 0 && !e.sgd) {  // nothing to write (cannot happen for scheduled tasks)
@@ -1049,9 +1120,9 @@ __device__ void data_warp(const LaunchArgs &a, const TreeParams &p, int role, in
     return;
   }
   switch (e.nin) {
-    case 1: lsu_nout<DT, 1, SGD, MAXT>(a, e, t, j, w, W, sh); break;
-    case 2: lsu_nout<DT, 2, SGD, MAXT>(a, e, t, j, w, W, sh); break;
-    default: lsu_nout<DT, 3, SGD, MAXT>(a, e, t, j, w, W, sh); break;
+    case 1: lsu_nout<DT, 1, SGD, MAXT>(a, e, t, j, w, W, sh, iw, iW); break;
+    case 2: lsu_nout<DT, 2, SGD, MAXT>(a, e, t, j, w, W, sh, iw, iW); break;
+    default: lsu_nout<DT, 3, SGD, MAXT>(a, e, t, j, w, W, sh, iw, iW); break;
   }
 }
 
@@ -1091,11 +1162,12 @@ __global__ void __launch_bounds__(MAXT, kMinBlocksPerSm) tree_allreduce_kernel(c
     else
       control_warp<SYS>(a, p, task.role, task.tree, task.channel, W, sh);
   } else if (warp < nctl) {
-    publish_warp<SYS>(a, p, task.role, task.tree, task.channel, W, sh);
+    publish_warp<SYS>(a, p, task.role, task.tree, task.channel, W, sh, task.half, task.halves);
   } else if (a.tma) {
     tma_data_warp<DT, SGD>(a, p, task.role, task.tree, task.channel, warp - nctl, W, sh, tma_ring);
   } else {
-    data_warp<DT, SGD, MAXT>(a, p, task.role, task.tree, task.channel, warp - nctl, W, sh);
+    data_warp<DT, SGD, MAXT>(a, p, task.role, task.tree, task.channel, warp - nctl, W, sh,
+                             task.half, task.halves);
   }
 }
 

@@ -738,3 +738,19 @@ def test_ll_gate_opens_after_landing(comm):
     for s, hi in zip(snaps, ends):
         assert torch.equal(s, ts[7][lo:hi])
         lo = hi
+
+
+@pytest.mark.parametrize("P,kind", [(8, "single"), (8, "double"), (4, "single"), (2, "single")])
+@pytest.mark.parametrize("overlap", [True, False])
+def test_parity_split_heads(comm, monkeypatch, P, kind, overlap):
+    """CCUBE_SPLIT_HEADS=1: the pipeline's head tasks on two CTAs per channel, the
+    halves publishing a monotone max of their joint progress — bit-exact vs the
+    oracle, several chunks, ragged tail, auto channels."""
+    monkeypatch.setenv("CCUBE_SPLIT_HEADS", "1")
+    chunk = 64 << 10
+    comm(P, kind, chunk, overlap=overlap)
+    count = 9 * chunk // 4 + 77
+    xs, outs = _run(P, kind, "float32", count, chunk)
+    ref = oar.reference(xs, kind, chunk, "float32")[0]
+    for r in range(P):
+        assert np.array_equal(outs[r], ref), f"rank {r}"
