@@ -122,6 +122,7 @@ struct Task {
   int16_t channel;   // kAllChannels for a pulled leaf
   int16_t half;      // 0, or 1 for the second CTA of a split task
   int16_t halves;    // 1, or 2 for a split task
+  int16_t head;      // 1: an UP task at the pipeline's head (children = pulled leaves)
 };
 
 struct LaunchArgs {

@@ -534,9 +534,9 @@ ccube_result_t get_tasks(int channels, int overlap, TaskTable **out) {
     return CCUBE_SUCCESS;
   }
   const PlanIn in = plan_in(0);
-  auto task = [](int i, int t, int role, int j, int half = 0, int halves = 1) {
+  auto task = [](int i, int t, int role, int j, int half = 0, int halves = 1, int head = 0) {
     return Task{(int16_t)i, (int16_t)t, (int16_t)role, (int16_t)j, (int16_t)half,
-                (int16_t)halves};
+                (int16_t)halves, (int16_t)head};
   };
   std::vector<Task> ts;
   for (int i = 0; i < g.nlocal; ++i) {
@@ -551,10 +551,11 @@ ccube_result_t get_tasks(int channels, int overlap, TaskTable **out) {
         continue;
       }
       const bool down = tr.nchild[r] > 0 && (!root || !overlap);
-      const bool head = split && plan_is_head(in, tr, r);
+      const bool is_head = plan_is_head(in, tr, r);
+      const bool head = split && is_head;
       for (int j = 0; j < channels; ++j) {
-        ts.push_back(task(i, t, kRoleUp, j, 0, head ? 2 : 1));
-        if (head) ts.push_back(task(i, t, kRoleUp, j, 1, 2));
+        ts.push_back(task(i, t, kRoleUp, j, 0, head ? 2 : 1, is_head));
+        if (head) ts.push_back(task(i, t, kRoleUp, j, 1, 2, is_head));
       }
       if (down)
         for (int j = 0; j < channels; ++j) ts.push_back(task(i, t, kRoleDown, j));

@@ -1143,10 +1143,11 @@ __global__ void __launch_bounds__(MAXT, kMinBlocksPerSm) tree_allreduce_kernel(c
   }
   const int nctl = a.split_control ? 2 : 1;  // control warps ahead of the data warps
   const int W = (blockDim.x >> 5) - nctl;
+  const bool tma = a.tma != 0;
   if (threadIdx.x == 0) {
     sh.ready = 0;
     sh.abort = 0;
-    if (a.tma) {
+    if (tma) {
       for (int s = 0; s < kTmaMaxStages; ++s) {
         mbar_init(&sh.full[s], 1);
         mbar_init(&sh.empty[s], W - 1);
@@ -1163,7 +1164,7 @@ __global__ void __launch_bounds__(MAXT, kMinBlocksPerSm) tree_allreduce_kernel(c
       control_warp<SYS>(a, p, task.role, task.tree, task.channel, W, sh);
   } else if (warp < nctl) {
     publish_warp<SYS>(a, p, task.role, task.tree, task.channel, W, sh, task.half, task.halves);
-  } else if (a.tma) {
+  } else if (tma) {
     tma_data_warp<DT, SGD>(a, p, task.role, task.tree, task.channel, warp - nctl, W, sh, tma_ring);
   } else {
     data_warp<DT, SGD, MAXT>(a, p, task.role, task.tree, task.channel, warp - nctl, W, sh,
