@@ -77,8 +77,9 @@ def parse(argv=None):
     p.add_argument("--iter-warmup", type=int, default=2)
     p.add_argument("--iter-channels", type=int, default=4,
                    help="loopback: AllReduce channels of the chained iteration")
-    p.add_argument("--iter-channels-multi", type=int, default=0,
-                   help="N>1: AllReduce channels of the chained iteration (0 = auto)")
+    p.add_argument("--iter-channels-multi", type=int, default=16,
+                   help="N>1: AllReduce channels of the chained iteration (0 = auto, which "
+                        "gives the AllReduce every SM and the forward nothing to overlap on)")
     p.add_argument("--iter-tree", choices=["single", "double", "rotated"], default="single")
     p.add_argument("--iter-rank", type=int, default=1,
                    help="loopback rank that hosts the model replica (1 = a leaf of tree 0)")
