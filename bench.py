@@ -633,7 +633,12 @@ def run_ccube(a):
     # ---- NVLink roofline instrument (N>1): the kernel's own peer-store path
     port_peak = None
     if multi and not a.no_port_peak:
-        pair, fan = ccube.measure_peer_bandwidth(64 << 20, 5)
+        try:
+            pair, fan = ccube.measure_peer_bandwidth(64 << 20, 5)
+        except Exception as e:  # noqa: BLE001 — reported; the roofline falls back
+            pair, fan = None, None
+            port_peak = {"error": repr(e)}
+    if multi and not a.no_port_peak and pair is not None:
         port_peak = {"pair_gbs": pair, "fanout_egress_gbs": fan,
                      "bytes_per_destination": 64 << 20,
                      "how": "ccube_measure_peer_bandwidth: 128-bit loads from local HBM, "
@@ -699,13 +704,19 @@ def run_ccube(a):
     if not a.no_extra:
         extra = {}
         for kind in [k for k in ("single", "double", "rotated") if k != a.tree]:
-            init(kind)
-            ms_k, tot_k = _time_steps(lambda: allreduce(bufs), restorer(bufs, pristine),
-                                      a.extra_steps, 3, stream, multi, hdev)
-            ok_k, _ = _ranks_identical(bufs, multi, None if shared else dev)
-            extra[kind] = _extra_line(P, kind, nbytes, tot_k / a.extra_steps, multi, port_peak,
-                                      ccube.get_info(), ok_k, a.workload, a.dtype)
-            ccube.finalize()
+            try:
+                init(kind)
+                try:
+                    ms_k, tot_k = _time_steps(lambda: allreduce(bufs), restorer(bufs, pristine),
+                                              a.extra_steps, 3, stream, multi, hdev)
+                    ok_k, _ = _ranks_identical(bufs, multi, None if shared else dev)
+                    extra[kind] = _extra_line(P, kind, nbytes, tot_k / a.extra_steps, multi,
+                                              port_peak, ccube.get_info(), ok_k, a.workload,
+                                              a.dtype)
+                finally:
+                    ccube.finalize()
+            except Exception as e:  # noqa: BLE001 — reported; the main line stands
+                extra[kind] = {"error": repr(e)}
         del bufs, pristine
         torch.cuda.empty_cache()
         if not a.max_elems:
@@ -714,14 +725,19 @@ def run_ccube(a):
             vp = [torch.randn(vcount, device=dev, generator=g).to(torch.bfloat16)
                   for _ in my_ranks]
             vb = [p.clone() for p in vp]
-            init("double")
-            ms_v, tot_v = _time_steps(lambda: allreduce(vb), restorer(vb, vp), a.extra_steps, 3,
-                                      stream, multi, hdev)
-            ok_v, _ = _ranks_identical(vb, multi, None if shared else dev)
-            extra["vgg16_bf16_double"] = _extra_line(P, "double", vcount * 2,
-                                                     tot_v / a.extra_steps, multi, port_peak,
-                                                     ccube.get_info(), ok_v, "vgg16", "bfloat16")
-            ccube.finalize()
+            try:
+                init("double")
+                try:
+                    ms_v, tot_v = _time_steps(lambda: allreduce(vb), restorer(vb, vp),
+                                              a.extra_steps, 3, stream, multi, hdev)
+                    ok_v, _ = _ranks_identical(vb, multi, None if shared else dev)
+                    extra["vgg16_bf16_double"] = _extra_line(
+                        P, "double", vcount * 2, tot_v / a.extra_steps, multi, port_peak,
+                        ccube.get_info(), ok_v, "vgg16", "bfloat16")
+                finally:
+                    ccube.finalize()
+            except Exception as e:  # noqa: BLE001 — reported; the main line stands
+                extra["vgg16_bf16_double"] = {"error": repr(e)}
             if multi and not a.no_nccl and not shared:
                 extra["vgg16_bf16_double"]["nccl"] = nccl_compare(a, dev, vb[0], vp[0],
                                                                   vcount * 2, P, stream)
@@ -781,7 +797,7 @@ def _nvlink_roofline(P, kind, nbytes, ms_step, port_peak):
     SURVEY §8(d)) over the kernel time, against the measured port peak."""
     port = max(_port_loads(P, kind)) * nbytes
     achieved = port / (ms_step / 1e3) / 1e9
-    if port_peak is not None:
+    if port_peak is not None and "fanout_egress_gbs" in port_peak:
         peak = max(port_peak["fanout_egress_gbs"][1:])
         src = "measured: ccube_measure_peer_bandwidth, best fan-out egress per GPU"
     else:

@@ -328,10 +328,13 @@ def set_overlap(on: bool) -> None:
 
 
 def set_channels(channels: int) -> None:
+    """Channels per tree (0 = auto).  Collective with several processes."""
     _check(lib().ccube_set_channels(channels), "ccube_set_channels")
 
 
 def set_threads(threads: int) -> None:
+    """Data threads per CTA (32..256, multiple of 32), or 0 = auto (the default: 6 data
+    warps when the channel slices hold >= 3 units of 2 KB, else 8)."""
     _check(lib().ccube_set_threads(threads), "ccube_set_threads")
 
 
