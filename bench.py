@@ -50,6 +50,8 @@ def parse(argv=None):
     p.add_argument("--datapath", choices=["auto", "tma", "lsu"], default=None,
                    help="data-warp datapath (default: the library's, CCUBE_DATAPATH)")
     p.add_argument("--e2e-steps", type=int, default=10)
+    p.add_argument("--e2e-copy-streams", type=int, default=2,
+                   help="e2e: streams (copy engines) per copy direction")
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--no-clocks", action="store_true")
@@ -585,26 +587,38 @@ def run_ccube(a):
     if not a.no_e2e:
         outs = [torch.empty_like(h).pin_memory() for h in host]
         sets = [bufs, [torch.empty_like(b) for b in bufs]]
-        dstream = torch.cuda.Stream()
         ev = lambda: torch.cuda.Event()  # noqa: E731
+        # the copies of one direction are spread over `ncs` streams (copy engines); the
+        # AllReduce runs on `stream` after every H2D stream of its step
+        ncs = max(1, min(a.e2e_copy_streams, len(host)))
+        h2d = [stream] + [torch.cuda.Stream() for _ in range(ncs - 1)]
+        d2h = [torch.cuda.Stream() for _ in range(ncs)]
         d2h_done = [None, None]
 
         def e2e_step(i):
             s_ = i % 2
-            if d2h_done[s_] is not None:          # step i-2's results are out of this set
-                stream.wait_event(d2h_done[s_])
-            with torch.cuda.stream(stream):
-                for b, h in zip(sets[s_], host):
-                    b.copy_(h, non_blocking=True)
+            for q, hs in enumerate(h2d):
+                if d2h_done[s_] is not None:      # step i-2's results are out of this set
+                    for e_ in d2h_done[s_]:
+                        hs.wait_event(e_)
+                with torch.cuda.stream(hs):
+                    for r in range(q, len(host), ncs):
+                        sets[s_][r].copy_(host[r], non_blocking=True)
+                if q:
+                    e_ = ev()
+                    e_.record(hs)
+                    stream.wait_event(e_)
             allreduce(sets[s_])
             k = ev()
             k.record(stream)
-            dstream.wait_event(k)
-            with torch.cuda.stream(dstream):
-                for o, b in zip(outs, sets[s_]):
-                    o.copy_(b, non_blocking=True)
-            d2h_done[s_] = ev()
-            d2h_done[s_].record(dstream)
+            d2h_done[s_] = []
+            for q, ds in enumerate(d2h):
+                ds.wait_event(k)
+                with torch.cuda.stream(ds):
+                    for r in range(q, len(host), ncs):
+                        outs[r].copy_(sets[s_][r], non_blocking=True)
+                d2h_done[s_].append(ev())
+                d2h_done[s_][-1].record(ds)
 
         for i in range(2):
             e2e_step(i)
@@ -615,7 +629,8 @@ def run_ccube(a):
         e0.record(stream)
         for i in range(a.e2e_steps):
             e2e_step(i)
-        stream.wait_stream(dstream)
+        for ds in d2h:
+            stream.wait_stream(ds)
         e1.record(stream)
         torch.cuda.synchronize()
         e2e_ms = e0.elapsed_time(e1) / a.e2e_steps
@@ -626,7 +641,8 @@ def run_ccube(a):
         e2e = {"value": ebw, "unit": "GB/s", "ms_per_step": e2e_ms,
                "h2d_bytes_per_step": nbytes * len(my_ranks),
                "d2h_bytes_per_step": nbytes * len(my_ranks), "steps": a.e2e_steps,
-               "pipelining": "two device buffer sets; step i's D2H overlaps step i+1's H2D",
+               "pipelining": f"two device buffer sets; step i's D2H overlaps step i+1's H2D; "
+                             f"each direction on {ncs} stream(s)",
                "ranks_identical": ok_e2e}
         del sets
 
