@@ -50,7 +50,7 @@ def parse(argv=None):
     p.add_argument("--datapath", choices=["auto", "tma", "lsu"], default=None,
                    help="data-warp datapath (default: the library's, CCUBE_DATAPATH)")
     p.add_argument("--e2e-steps", type=int, default=10)
-    p.add_argument("--e2e-copy-streams", type=int, default=2,
+    p.add_argument("--e2e-copy-streams", type=int, default=1,
                    help="e2e: streams (copy engines) per copy direction")
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-cpu-baseline", action="store_true")
