@@ -593,6 +593,10 @@ ccube_result_t ll_impl(Registration *R, size_t count, ccube_dtype_t dtype, uint6
   const int threads = 512;
   uint64_t ctas = (lines + 4 * threads - 1) / (4 * threads);  // <= 4 lines per thread
   if (ctas > 16) ctas = 16;
+  // every LL CTA polls lines other CTAs produce: all must be co-resident (one 512-thread
+  // CTA per SM is always available to this kernel's 86-register threads)
+  const uint64_t per_rank_max = static_cast<uint64_t>(g.sm_count / g.nlocal);
+  if (ctas > per_rank_max) ctas = per_rank_max > 0 ? per_rank_max : 1;
   a.ctas = static_cast<int>(ctas);
   a.count = count;
   a.epoch = g.ll_epoch + 1;
