@@ -327,3 +327,21 @@ def test_measure_peer_bandwidth_runs_collectively():
         for j in range(3):
             assert (pair0[i][j] > 0) == (i != j)
     assert fan0[0] == 0 and all(f > 0 for f in fan0[1:])
+
+
+@pytest.mark.parametrize("kind,count", [("double", 70_001), ("single", 3_001)])
+def test_multiprocess_ipc_parity_p8(kind, count):
+    """Eight processes (the target's P): the double tree chunked (16 KiB chunks,
+    interior ranks in one tree and leaves in the other, every edge PUSH over IPC)
+    and a one-chunk message on the LL kernel, bit-exact to the oracle with the
+    gates checked, as in test_multiprocess_ipc_parity."""
+    from oracle import allreduce as oar
+    from paper_conf_hpca_sanghoonsk23_b200 import inputs
+    world, dtype, chunk = 8, "float32", 16 << 10
+    res = _run(world, kind, dtype, count, chunk)
+    xs = [inputs.gradients(r, count, dtype) for r in range(world)]
+    ref = oar.reference(xs, kind, chunk, dtype)[0]
+    for rank, err, out, early in res:
+        assert err == "", f"rank {rank}: {err}"
+        assert np.array_equal(out, ref), f"rank {rank} differs from the oracle"
+        assert not early, f"rank {rank}: a gate opened before its layer landed"

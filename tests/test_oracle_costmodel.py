@@ -59,3 +59,26 @@ def test_port_ceiling_table():
     assert max(costmodel.port_loads(8, "single", 1.0)) == 3
     t0 = trees.tree0(8)
     assert costmodel.port_loads(8, "single", 1.0)[0] == len(t0.children[0])
+
+
+@pytest.mark.parametrize("P", [2, 3, 4, 5, 8, 16])
+def test_ring_beta_term_is_the_bandwidth_optimal_port_load(P):
+    """Eq 2's bandwidth term 2((P-1)/P) beta N is the per-rank load of a ring; it must
+    equal, independently, the per-rank port load of the rotated tree set computed
+    from the trees (every rank holds every position once, R17) — and lower-bound
+    every tree shape's busiest port."""
+    ring_beta = costmodel.t_ring(P, N, 0.0, B) / B          # alpha = 0: bytes per rank
+    rot = costmodel.port_loads(P, "rotated", N)
+    assert all(math.isclose(x, ring_beta) for x in rot)
+    for kind in ("single", "double"):
+        assert max(costmodel.port_loads(P, kind, N)) >= ring_beta * (1 - 1e-12)
+
+
+@pytest.mark.parametrize("P", [2, 4, 8])
+def test_allgather_is_the_ring_half(P):
+    """Eq 1 vs eq 2 at any P: the ring AllReduce is a reduce-scatter plus an
+    all-gather of P-1 steps each, so t_ring = 2 t_allgather for every (alpha, beta);
+    with beta = 0 it is 2(P-1) alpha (P-1 dependent steps per phase)."""
+    assert math.isclose(costmodel.t_ring(P, N, A, B), 2 * costmodel.t_allgather(P, N, A, B))
+    assert math.isclose(costmodel.t_ring(P, N, A, 0.0), 2 * (P - 1) * A)
+    assert math.isclose(costmodel.t_allgather(P, N, 0.0, B), (P - 1) / P * N * B)
