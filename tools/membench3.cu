@@ -4,7 +4,10 @@
 //   lsu256 : the same with 256-bit vectors (ld/st.global.v8.u32, sm_100a);
 //   occ128 : the same loop at full occupancy (8 CTAs of 8 warps per SM);
 // for the stream shapes of the tree tasks: copy 1->1 / 1->2 (DOWN), 2->2 (C1 root),
-// 3->1 (interior UP).  gbs counts every byte read + written (best of 5 launches).
+// 3->1 (interior UP); and fold8, the loopback AllReduce's algorithmic floor done in
+// one dependency-free pass (8 inputs read once, their fixed-order sum written to 8
+// outputs) — the practical ceiling for any loopback AllReduce of that size.  gbs
+// counts every byte read + written (best of 5 launches).  Argument: MiB per buffer.
 //
 //   nvcc -gencode arch=compute_100a,code=sm_100a -O3 -std=c++17 -o membench3 tools/membench3.cu
 #include <cuda_runtime.h>
@@ -21,8 +24,8 @@
   } while (0)
 
 struct Bufs {
-  const char *src[3];
-  char *dst[3];
+  const char *src[8];
+  char *dst[8];
 };
 
 struct V8 {
@@ -113,6 +116,33 @@ __global__ void __launch_bounds__(256, 8) k_occ(Bufs b, size_t bytes) {
   stream<NIN, NOUT, U, VB>(b, bytes);
 }
 
+// The loopback AllReduce's floor as one pass: every rank's input read once, the
+// fixed-order sum computed in registers, every rank's output written once (2*P*N
+// bytes, P = 8) — an upper bound for any loopback AllReduce of this size.
+template <int U>
+__global__ void __launch_bounds__(256, 2) k_fold8(Bufs b, size_t bytes) {
+  const int lane = threadIdx.x & 31;
+  const size_t gw = (blockIdx.x * (size_t)blockDim.x + threadIdx.x) >> 5;
+  const size_t nw = (gridDim.x * (size_t)blockDim.x) >> 5;
+  const size_t blk = 512ull * U;
+  for (size_t G = gw; G < bytes / blk; G += nw) {
+    const size_t off = G * blk + lane * 16;
+    uint4 x[U][8];
+#pragma unroll
+    for (int u = 0; u < U; ++u)
+#pragma unroll
+      for (int q = 0; q < 8; ++q) x[u][q] = Vec<16>::ld(b.src[q] + off + 512 * u);
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      uint4 r = x[u][0];
+#pragma unroll
+      for (int q = 1; q < 8; ++q) r = Vec<16>::add(r, x[u][q]);
+#pragma unroll
+      for (int q = 0; q < 8; ++q) Vec<16>::st(b.dst[q] + off + 512 * u, r);
+    }
+  }
+}
+
 size_t g_bytes;
 int g_sms;
 
@@ -149,16 +179,20 @@ int run(const char *name, K kern, int nin, int nout, int u, int vb, int grid, Bu
 int main(int argc, char **argv) {
   CK(cudaDeviceGetAttribute(&g_sms, cudaDevAttrMultiProcessorCount, 0));
   g_bytes = (argc > 1 ? (size_t)atol(argv[1]) : 256) << 20;
-  char *p[6];
-  for (int i = 0; i < 6; ++i) {
+  char *p[16];
+  for (int i = 0; i < 16; ++i) {
     CK(cudaMalloc(&p[i], g_bytes));
     CK(cudaMemset(p[i], 0, g_bytes));
   }
   Bufs b;
-  for (int i = 0; i < 3; ++i) {
+  for (int i = 0; i < 8; ++i) {
     b.src[i] = p[i];
-    b.dst[i] = p[3 + i];
+    b.dst[i] = p[8 + i];
   }
+  run("fold8", k_fold8<1>, 8, 8, 1, 16, 2 * g_sms, b);
+  run("fold8", k_fold8<2>, 8, 8, 2, 16, 2 * g_sms, b);
+  run("fold8", k_fold8<1>, 8, 8, 1, 16, 4 * g_sms, b);
+  for (int i = 0; i < 3; ++i) b.dst[i] = p[3 + i];
   RUN3(1, 1, 4)
   RUN3(1, 1, 8)
   RUN3(1, 2, 4)
