@@ -55,6 +55,12 @@ namespace {
 #ifndef CCUBE_U_COMBINE_192
 #define CCUBE_U_COMBINE_192 8  // <= 192 threads (4 data warps)
 #endif
+#ifndef CCUBE_DONE_INIT
+#define CCUBE_DONE_INIT 1  // data warps report their first block's chunk at start
+#endif
+#ifndef CCUBE_OWN_FIRST
+#define CCUBE_OWN_FIRST 1  // combines load their own input before the readiness wait
+#endif
 #ifndef CCUBE_U_COPY_S
 #define CCUBE_U_COPY_S 4
 #endif
@@ -820,8 +826,31 @@ __device__ void lsu_stream(const LaunchArgs &a, const Endpoints &e, int t, int j
 #pragma unroll
   for (int q = 0; q < NOUT; ++q) dpol[q] = (e.keep >> q) & 1u ? pol.last : pol.first;
   BlockIter it = iter_begin<kSeg>(g, iw);  // iw / iW: this warp among the task's CTAs
+  // "done" = the chunk of my next block: I have no block in the chunks before my first
+  // one, so say so now — otherwise chunk 0 is released only once every warp (including
+  // those whose first block lies in chunk 1 or 2) has finished its first block, i.e.
+  // each hop of the pipeline's fill would wait for two more upstream chunks.
+  if (CCUBE_DONE_INIT && it.k > 0) {
+    if (lane == 0) st_release_cta(&sh.done[w], it.k);
+    done_reported = it.k;
+  }
+  // A combine (UP with children) reads my own input first: it is in my buffer from
+  // the start, so its loads go out before the wait for the children's partials and
+  // only the partials' (L2) latency stays on the hop's critical path.
+  constexpr bool kOwnFirst = CCUBE_OWN_FIRST && NIN >= 2 && !SGD;
   while (it.k < g.K) {
     const uint32_t k = it.k;
+    const uint32_t b0 = it.s * kSeg;
+    const uint64_t off = it.sl.off + b0;
+    const uint32_t len = min(kSeg, it.sl.len - b0);
+    const uint32_t nvec = len / 16;
+    uint4 x[U][NIN];
+    uint4 wv[SGD ? U : 1];
+    if constexpr (kOwnFirst) {
+#pragma unroll
+      for (int u = 0; u < U; ++u)
+        if (lane + 32u * u < nvec) x[u][0] = ld_hint(e.src[0] + off + lane * 16 + 512u * u, pol.first);
+    }
     if (k >= ready) {
       uint64_t r = 0;
       if (lane == 0) {  // upstream not there yet: back off so busy warps get the issue slots
@@ -833,17 +862,11 @@ __device__ void lsu_stream(const LaunchArgs &a, const Endpoints &e, int t, int j
       if (r <= k) return;  // aborted
       ready = r;
     }
-    const uint32_t b0 = it.s * kSeg;
-    const uint64_t off = it.sl.off + b0;
-    const uint32_t len = min(kSeg, it.sl.len - b0);
-    const uint32_t nvec = len / 16;
-    uint4 x[U][NIN];
-    uint4 wv[SGD ? U : 1];
 #pragma unroll
     for (int u = 0; u < U; ++u) {
       if (lane + 32u * u < nvec) {
 #pragma unroll
-        for (int q = 0; q < NIN; ++q)
+        for (int q = kOwnFirst ? 1 : 0; q < NIN; ++q)
           x[u][q] = ld_hint(e.src[q] + off + lane * 16 + 512u * u, pol.first);
         if constexpr (SGD) wv[u] = ld_hint(e.w + off + lane * 16 + 512u * u, pol.first);
       }
