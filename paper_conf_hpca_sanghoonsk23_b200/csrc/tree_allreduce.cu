@@ -156,6 +156,14 @@ __device__ __forceinline__ float bf_hi(uint32_t w) { return __uint_as_float(w & 
 __device__ __forceinline__ uint32_t bf_round(float f) {
   return static_cast<uint32_t>(__bfloat16_as_ushort(__float2bfloat16_rn(f)));
 }
+// Both halves of a word at once: cvt.rn.bf16x2.f32 rounds each input to nearest-even
+// exactly as cvt.rn.bf16.f32 does (no FTZ), in one packed conversion (F2FP.PACK_AB)
+// instead of two F2F conversions and a byte permute.
+__device__ __forceinline__ uint32_t bf_pack(float lo, float hi) {
+  uint32_t r;
+  asm("cvt.rn.bf16x2.f32 %0, %1, %2;" : "=r"(r) : "f"(hi), "f"(lo));
+  return r;
+}
 
 template <int DT>
 struct Combine;
@@ -217,7 +225,7 @@ struct Combine<kBFloat16> {
       lo = __fadd_rn(lo, bf_lo(w[i]));
       hi = __fadd_rn(hi, bf_hi(w[i]));
     }
-    return bf_round(lo) | (bf_round(hi) << 16);
+    return bf_pack(lo, hi);
   }
   template <int N>
   __device__ __forceinline__ static uint4 vec(const uint4 (&v)[N]) {
@@ -1316,7 +1324,7 @@ __device__ __forceinline__ uint32_t ll_combine(uint32_t own, uint32_t c0, uint32
       lo = __fadd_rn(lo, bf_lo(c1));
       hi = __fadd_rn(hi, bf_hi(c1));
     }
-    return bf_round(lo) | (bf_round(hi) << 16);
+    return bf_pack(lo, hi);
   }
 }
 
