@@ -210,8 +210,9 @@ CCUBE_API ccube_result_t ccube_set_threads(int threads);
  * ranks must agree).  LSU: each data warp keeps its own 128-bit loads in flight in
  * registers.  TMA: one data warp streams every source block into a 96 KB
  * shared-memory ring with cp.async.bulk and the other data warps combine from it
- * (needs >= 2 data warps; with one the LSU path runs).  AUTO (default): TMA for the
- * rotated tree set, LSU otherwise (measured).  CCUBE_DATAPATH env
+ * (needs >= 2 data warps; with one the LSU path runs).  AUTO (default): LSU for every
+ * tree kind (round 1 chose TMA for the rotated set; with its leaf-group CTAs LSU is
+ * faster there too, measured).  CCUBE_DATAPATH env
  * (0 / 1) sets the initial value.  Errors: NOT_INITIALIZED, INVALID_ARG. */
 #define CCUBE_DATAPATH_AUTO (-1)
 #define CCUBE_DATAPATH_LSU 0

@@ -119,9 +119,10 @@ struct Task {
   int16_t local_rank;
   int16_t tree;
   int16_t role;
-  int16_t channel;   // kAllChannels for a pulled leaf
-  int16_t half;      // 0, or 1 for the second CTA of a split task
-  int16_t halves;    // 1, or 2 for a split task
+  int16_t channel;   // kAllChannels for a pulled leaf (and the leaf-group CTA)
+  int16_t half;      // 0, or 1 for the second CTA of a split task; leaf group: the
+                     // table index of its first pulled leaf
+  int16_t halves;    // 1, or 2 for a split task; leaf group: its number of leaves
   int16_t head;      // 1: an UP task at the pipeline's head (children = pulled leaves)
 };
 

@@ -24,18 +24,20 @@ int plan_tasks_of_proc(const PlanIn &in, int proc, int J) {
   int n = 0;
   for (int i = 0; i < in.nlocal; ++i) {
     const int r = proc * in.nlocal + i;
+    bool pulled = false;  // every pulled leaf of rank r shares one CTA
     for (int t = 0; t < in.ntrees; ++t) {
       const Tree &tr = in.trees[t];
       const bool root = tr.parent[r] < 0;
       const bool leaf = !root && tr.nchild[r] == 0;
       if (leaf && in.sgd) n += J;  // a leaf's fused SGD step (f2)
       if (leaf && plan_edge_is_pull(in.transport, in.nlocal, r, tr.parent[r])) {
-        n += 1;  // a pulled leaf: one CTA publishes every channel
+        pulled = true;  // a pulled leaf: the rank's leaf-group CTA publishes every channel
         continue;
       }
       n += (in.split_heads && plan_is_head(in, tr, r)) ? 2 * J : J;  // UP
       if (tr.nchild[r] > 0 && (!root || !in.overlap)) n += J;  // DOWN
     }
+    if (pulled) n += 1;
   }
   return n;
 }

@@ -37,7 +37,10 @@ bool plan_is_head(const PlanIn &in, const Tree &tr, int r);
 // both ranks live in the same process (same GPU) under AUTO; PUSH otherwise.
 bool plan_edge_is_pull(int transport, int nlocal, int child, int parent);
 
-// CTAs process `proc` launches with J channels (the task table of runtime.cc).
+// CTAs process `proc` launches with J channels (the task table of runtime.cc): J
+// per UP / DOWN / UPDATE task, plus ONE leaf-group CTA per rank for all the trees in
+// which it is a pulled leaf (a pulled leaf only publishes its heads and waits for its
+// result).
 int plan_tasks_of_proc(const PlanIn &in, int proc, int J);
 
 // Maximum over every process of the communicator.

@@ -304,11 +304,13 @@ bool edge_is_pull(int child, int parent) {
   return plan_edge_is_pull(g.transport, g.nlocal, child, parent);
 }
 
-// The TMA datapath is chosen by the datapath setting and the tree kind (AUTO: TMA
-// for the rotated set); the split of the pipeline's head tasks runs on the LSU path
-// with the two control warps, without the fused update.
+// The TMA datapath runs only when chosen (AUTO = LSU: round 1's AUTO picked TMA for
+// the rotated set, whose slices were long at J = 4; at J = 5 with the leaf-group
+// CTAs, LSU measured faster at P = 2 / 4 / 8).  The split of the
+// pipeline's head tasks runs on the LSU path with the two control warps, without the
+// fused update.
 bool want_tma() {
-  return g.datapath == CCUBE_DATAPATH_TMA || (g.datapath == CCUBE_DATAPATH_AUTO && g.ntrees > 2);
+  return g.datapath == CCUBE_DATAPATH_TMA;
 }
 bool split_heads_now() {
   return g.split_heads && !g.sgd && !want_tma() && g.split_control;
@@ -538,16 +540,17 @@ ccube_result_t get_tasks(int channels, int overlap, TaskTable **out) {
     return Task{(int16_t)i, (int16_t)t, (int16_t)role, (int16_t)j, (int16_t)half,
                 (int16_t)halves, (int16_t)head};
   };
-  std::vector<Task> ts;
+  std::vector<Task> ts, leaves;
   for (int i = 0; i < g.nlocal; ++i) {
     const int r = g.rank0 + i;
+    const size_t first_leaf = leaves.size();
     for (int t = 0; t < g.ntrees; ++t) {
       const Tree &tr = g.trees[t];
       const bool root = tr.parent[r] < 0;
       if (!root && tr.nchild[r] == 0 && g.sgd)  // a leaf's fused SGD step (f2)
         for (int j = 0; j < channels; ++j) ts.push_back(task(i, t, kRoleUpdate, j));
       if (!root && tr.nchild[r] == 0 && edge_is_pull(r, tr.parent[r])) {
-        ts.push_back(task(i, t, kRoleUp, kAllChannels));
+        leaves.push_back(task(i, t, kRoleUp, kAllChannels));
         continue;
       }
       const bool down = tr.nchild[r] > 0 && (!root || !overlap);
@@ -560,10 +563,19 @@ ccube_result_t get_tasks(int channels, int overlap, TaskTable **out) {
       if (down)
         for (int j = 0; j < channels; ++j) ts.push_back(task(i, t, kRoleDown, j));
     }
+    // One leaf-group CTA per rank serves the trees in which the rank is a pulled leaf
+    // (one tree for the single and double tree, P/2 of the rotated set's P); its
+    // leaves' entries follow the grid in the table (`half` is fixed up below).
+    if (leaves.size() > first_leaf)
+      ts.push_back(task(i, 0, kRoleUp, kAllChannels, static_cast<int>(first_leaf),
+                        static_cast<int>(leaves.size() - first_leaf)));
   }
   order_tasks(ts);
+  for (Task &x : ts)
+    if (x.channel == kAllChannels) x.half = static_cast<int16_t>(x.half + ts.size());
   TaskTable tt;
   tt.n = static_cast<int>(ts.size());
+  ts.insert(ts.end(), leaves.begin(), leaves.end());
   CUDA_TRY(cudaMalloc(&tt.d_tasks, sizeof(Task) * ts.size()));
   CUDA_TRY(cudaMemcpy(tt.d_tasks, ts.data(), sizeof(Task) * ts.size(), cudaMemcpyHostToDevice));
   g.tasks[key] = tt;
@@ -684,8 +696,6 @@ ccube_result_t allreduce_impl(void *const *bufs, size_t count, ccube_dtype_t dty
   // all CTAs spin on each other: they must be co-resident
   const int nctl = g.split_control ? 2 : 1;
   // the TMA datapath needs a producer and at least one consumer data warp
-  // (AUTO: TMA for the rotated tree set, whose P trees leave few channels and long
-  // slices per chunk; the register-staged LSU path for the single and double tree)
   const bool tma_wanted = want_tma();
   // co-resident CTAs per GPU for a CTA of `data` data threads (occupancy, cached)
   auto capacity = [&](int data, int *cap_out, int *tma_out) -> ccube_result_t {

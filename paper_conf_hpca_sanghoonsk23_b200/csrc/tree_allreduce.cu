@@ -613,22 +613,32 @@ __device__ __forceinline__ void leaf_wait(const LaunchArgs &a, const TreeParams 
   }
 }
 
-// A leaf on a PULL edge: its input already sits where the parent reads it.  One
-// warp publishes every channel's head at once and waits for the result.
+// Leaves on PULL edges: their inputs already sit where the parents read them.  One
+// CTA per rank (the leaf group, task entries [first, first + n) after the grid)
+// serves every tree in which the rank is a pulled leaf: its first warp publishes
+// every such leaf's head on every channel at once, then waits until the rank's
+// results have landed (the kernel completes only then).  All heads go out before
+// any wait: a leaf's result in one tree may need its input in another.
 template <bool SYS>
-__device__ void pulled_leaf(const LaunchArgs &a, const TreeParams &p, int t) {
+__device__ void pulled_leaves(const LaunchArgs &a, int first, int n) {
   const int lane = threadIdx.x & 31;
-  const uint32_t K = a.K[t];
-  const uint64_t base = a.base[t];
+  const int J = static_cast<int>(a.nchannels);
   fence_release<SYS>();
-  for (int j = lane; j < static_cast<int>(a.nchannels); j += 32)
-    st_relaxed<SYS>(p.head_out + j * kFlagStrideU64, base + K);
-  for (int j = lane; j < static_cast<int>(a.nchannels); j += 32) {
+  for (int x = lane; x < n * J; x += 32) {
+    const Task &l = a.tasks[first + x / J];
+    const TreeParams &p = a.params[l.local_rank * a.ntrees + l.tree];
+    st_relaxed<SYS>(p.head_out + (x % J) * kFlagStrideU64, a.base[l.tree] + a.K[l.tree]);
+  }
+  for (int x = lane; x < n * J; x += 32) {
+    const Task &l = a.tasks[first + x / J];
+    const TreeParams &p = a.params[l.local_rank * a.ntrees + l.tree];
+    const uint64_t target = a.base[l.tree] + a.K[l.tree];
+    uint64_t *enq = p.enq + (x % J) * kFlagStrideU64;
     Watch wd;
     watch_reset(wd);
-    while (ld_acquire<SYS>(p.enq + j * kFlagStrideU64) < base + K) {
-      if (!watch_tick(wd, a, base + K, 0)) {
-        st_relaxed<SYS>(p.enq + j * kFlagStrideU64, ~0ull);
+    while (ld_acquire<SYS>(enq) < target) {
+      if (!watch_tick(wd, a, target, 0)) {
+        st_relaxed<SYS>(enq, ~0ull);
         break;
       }
     }
@@ -1168,8 +1178,8 @@ __global__ void __launch_bounds__(MAXT, kMinBlocksPerSm) tree_allreduce_kernel(c
   const Task task = a.tasks[blockIdx.x];
   const TreeParams &p = a.params[task.local_rank * a.ntrees + task.tree];
   const int warp = threadIdx.x >> 5;
-  if (task.channel == kAllChannels) {
-    if (warp == 0) pulled_leaf<SYS>(a, p, task.tree);
+  if (task.channel == kAllChannels) {  // the leaf group
+    if (warp == 0) pulled_leaves<SYS>(a, task.half, task.halves);
     return;
   }
   const int nctl = a.split_control ? 2 : 1;  // control warps ahead of the data warps

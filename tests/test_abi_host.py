@@ -137,21 +137,23 @@ def test_gloo_bootstrap_detects_mismatch_ws2():
 
 def _py_tasks(P, kind, nlocal, proc, J, overlap):
     """Independent restatement of the task table: per rank and tree, UP on J channels,
-    DOWN on J channels at interior nodes (and at the root in B), a pulled leaf (same
-    process as its parent) one CTA."""
+    DOWN on J channels at interior nodes (and at the root in B); a rank that is a
+    pulled leaf (same process as its parent) in any tree adds one leaf-group CTA."""
     T = {"single": 1, "double": 2, "rotated": P}[kind]
     n = 0
     for r in range(proc * nlocal, (proc + 1) * nlocal):
+        pulled = False
         for t in range(T):
             par = ccube.tree_parents(P, kind, t)
             nch = sum(1 for u in range(P) if par[u] == r)
             root = par[r] < 0
             if not root and nch == 0 and par[r] // nlocal == r // nlocal:
-                n += 1
+                pulled = True
                 continue
             n += J
             if nch > 0 and (not root or not overlap):
                 n += J
+        n += 1 if pulled else 0
     return n
 
 
@@ -211,7 +213,11 @@ def test_plan_launch_loopback_and_explicit():
     # loopback: one process hosts every rank
     j, n, m = ccube.plan_launch(8, "single", 8, 0, 102_228_128, 256 << 10, 1, 0, 296)
     assert n == m == _py_tasks(8, "single", 8, 0, j, 1) <= 296
-    assert j == 41   # 7 J + 4 pulled leaves <= 296 (the round-1 bench geometry)
+    assert j == 41   # 7 J + 4 leaf-group CTAs (one per leaf rank) <= 296
+    # the double tree: 14 J + 8 <= 296 -> 20; the rotated set at P = 8: 56 J + 8 -> 5
+    # (round 1 spent one CTA per pulled leaf and tree: 56 J + 32 -> 4)
+    assert ccube.plan_launch(8, "double", 8, 0, 102_228_128, 256 << 10, 1, 0, 296)[0] == 20
+    assert ccube.plan_launch(8, "rotated", 8, 0, 102_228_128, 256 << 10, 1, 0, 296)[0] == 5
     # explicit channels are returned as given
     assert ccube.plan_launch(4, "double", 1, 2, 1 << 20, 0, 1, 7, 296)[0] == 7
     with pytest.raises(ccube.CCubeError) as e:

@@ -345,3 +345,22 @@ def test_multiprocess_ipc_parity_p8(kind, count):
         assert err == "", f"rank {rank}: {err}"
         assert np.array_equal(out, ref), f"rank {rank} differs from the oracle"
         assert not early, f"rank {rank}: a gate opened before its layer landed"
+
+
+@pytest.mark.parametrize("world,kind", [(4, "double"), (3, "single"), (4, "rotated")])
+def test_multiprocess_pull_transport(monkeypatch, world, kind):
+    """Every edge PULL across processes (CCUBE_TRANSPORT=2): a parent reads its
+    children's partials in place over IPC, so each leaf process runs its pulled
+    leaves on its leaf-group CTA (heads published at once, results awaited at .sys
+    scope).  Bit-exact vs the oracle, gates included."""
+    from oracle import allreduce as oar
+    from paper_conf_hpca_sanghoonsk23_b200 import inputs
+    monkeypatch.setenv("CCUBE_TRANSPORT", "2")
+    dtype, count, chunk = "float32", 50_001, 16 << 10
+    res = _run(world, kind, dtype, count, chunk)
+    xs = [inputs.gradients(r, count, dtype) for r in range(world)]
+    ref = oar.reference(xs, kind, chunk, dtype)[0]
+    for rank, err, out, early in res:
+        assert err == "", f"rank {rank}: {err}"
+        assert np.array_equal(out, ref), f"rank {rank} differs from the oracle"
+        assert not early, f"rank {rank}: a gate opened before its layer landed"
