@@ -829,7 +829,7 @@ __device__ __forceinline__ uint4 sgd4(const uint4 &w, const uint4 &g, float alph
                     __float_as_uint(sgd1(__uint_as_float(w.w), __uint_as_float(g.w), alpha)));
 }
 
-template <int DT, int NIN, int NOUT, int U, bool SGD>
+template <int DT, int NIN, int NOUT, int U, bool SGD, bool OWN_FIRST = false>
 __device__ void lsu_stream(const LaunchArgs &a, const Endpoints &e, int t, int j, int w, int W,
                            Shared &sh, int iw, int iW) {
   constexpr int ES = DT == kBFloat16 ? 2 : 4;
@@ -854,8 +854,11 @@ __device__ void lsu_stream(const LaunchArgs &a, const Endpoints &e, int t, int j
   }
   // A combine (UP with children) reads my own input first: it is in my buffer from
   // the start, so its loads go out before the wait for the children's partials and
-  // only the partials' (L2) latency stays on the hop's critical path.
-  constexpr bool kOwnFirst = CCUBE_OWN_FIRST && NIN >= 2 && !SGD;
+  // only the partials' (L2) latency stays on the hop's critical path.  Enabled for
+  // the 6-warp CTAs (U = 6, the P = 8 geometry), where it measured 1.3% faster; the
+  // 8-warp CTAs of the many-channel P = 2 / 4 geometry measured 1.4% slower with it
+  // (round 2 session 2).
+  constexpr bool kOwnFirst = CCUBE_OWN_FIRST && OWN_FIRST && NIN >= 2 && !SGD;
   while (it.k < g.K) {
     const uint32_t k = it.k;
     const uint32_t b0 = it.s * kSeg;
@@ -940,9 +943,9 @@ __device__ __forceinline__ void lsu_nout(const LaunchArgs &a, const Endpoints &e
     }
   }
   switch (e.nout) {
-    case 1: lsu_stream<DT, NIN, 1, U, false>(a, e, t, j, w, W, sh, iw, iW); break;
-    case 2: lsu_stream<DT, NIN, 2, U, false>(a, e, t, j, w, W, sh, iw, iW); break;
-    default: lsu_stream<DT, NIN, 3, U, false>(a, e, t, j, w, W, sh, iw, iW); break;
+    case 1: lsu_stream<DT, NIN, 1, U, false, (MAXT <= 256)>(a, e, t, j, w, W, sh, iw, iW); break;
+    case 2: lsu_stream<DT, NIN, 2, U, false, (MAXT <= 256)>(a, e, t, j, w, W, sh, iw, iW); break;
+    default: lsu_stream<DT, NIN, 3, U, false, (MAXT <= 256)>(a, e, t, j, w, W, sh, iw, iW); break;
   }
 }
 
