@@ -788,6 +788,7 @@ def run_ccube(a):
             "gpu_launches": a.steps * (2 if multi else 1),
             "ranks_identical": ok,
             "ms_per_step_p10_p50_p90": [float(np.percentile(ms, q)) for q in (10, 50, 90)],
+            "ms_per_step_max": float(np.max(ms)),
             "iteration": iteration,
         }
         if multi:

@@ -173,7 +173,8 @@ struct Comm {
   int l2_hints = 1;
   int datapath = CCUBE_DATAPATH_AUTO;  // CCUBE_DATAPATH env / ccube_set_datapath
   int last_tma = 0;
-  int split_control = 1;              // CCUBE_SPLIT_CONTROL env: poll and publish warps
+  int split_control = -1;             // CCUBE_SPLIT_CONTROL env: 1 poll + publish warps,
+                                      // 0 one control warp, -1 auto (per call)
   int backoff_ns = 64;                // CCUBE_BACKOFF_NS env: data warps' spin back-off
   int task_order = 0;                 // CCUBE_TASK_ORDER env: block -> task placement
   int debug_nodep = 0;                // CCUBE_DEBUG_NODEP env: timing experiments only
@@ -313,7 +314,7 @@ bool want_tma() {
   return g.datapath == CCUBE_DATAPATH_TMA;
 }
 bool split_heads_now() {
-  return g.split_heads && !g.sgd && !want_tma() && g.split_control;
+  return g.split_heads && !g.sgd && !want_tma() && g.split_control != 0;
 }
 
 PlanIn plan_in(uint64_t bytes) {
@@ -694,7 +695,7 @@ ccube_result_t allreduce_impl(void *const *bufs, size_t count, ccube_dtype_t dty
   if (K > 0xffffffffull) return fail(CCUBE_ERR_INVALID_ARG, "too many chunks");
 
   // all CTAs spin on each other: they must be co-resident
-  const int nctl = g.split_control ? 2 : 1;
+  int nctl = g.split_control == 0 ? 1 : 2;  // AUTO may drop to 1 below
   // the TMA datapath needs a producer and at least one consumer data warp
   const bool tma_wanted = want_tma();
   // co-resident CTAs per GPU for a CTA of `data` data threads (occupancy, cached)
@@ -723,16 +724,29 @@ ccube_result_t allreduce_impl(void *const *bufs, size_t count, ccube_dtype_t dty
   const PlanIn in = plan_in(bytes);
   int data_threads = g.threads, cap = 0, tma = 0;
   if (data_threads == 0) {
-    // auto CTA size: 6 data warps with 6 vectors in flight per lane and source (3 KB
+    // auto CTA size: 256-thread CTAs with 6 vectors in flight per lane and source (3 KB
     // blocks) when every channel's slice of a chunk holds >= 3 units of 2 KB, so the
     // 3 KB blocks tile it; 8 data warps with 2 KB blocks when the slices are short
     // (many channels: P = 2 / 4), where fewer warps would mean fewer bytes in flight
-    // (round 2).  Deterministic in agreed quantities, like J.
-    CC_TRY(capacity(kDefaultDataThreads, &cap, &tma));
+    // (round 2).  In the 256-thread case AUTO control (CCUBE_SPLIT_CONTROL
+    // unset) runs ONE control warp and 7 data warps instead of 2 + 6: the data warps'
+    // registers are the bytes in flight, and the extra warp outweighs the poll round
+    // trip a release may now wait behind (P = 8: single 0.3191 -> 0.3166 ms, double
+    // 0.3236 -> 0.3141 ms, round 2 session 2).  Deterministic in agreed
+    // quantities, like J.
+    CC_TRY(capacity(kDefaultDataThreads, &cap, &tma));  // a 256-thread CTA (nctl = 2)
     const int J0 = g.channels ? g.channels : plan_auto_channels(in, cap);
     const uint64_t first = bytes < g.chunk_bytes ? bytes : g.chunk_bytes;
     const uint64_t units = (first + 2047) / 2048;
-    data_threads = units >= 3ull * J0 ? kDefaultDataThreads : 256;
+    if (units >= 3ull * J0) {
+      data_threads = kDefaultDataThreads;
+      if (g.split_control < 0 && !split_heads_now()) {
+        nctl = 1;
+        data_threads += 32;  // the same 256-thread CTA
+      }
+    } else {
+      data_threads = 256;
+    }
   }
   CC_TRY(capacity(data_threads, &cap, &tma));
   const int cta_threads = data_threads + 32 * nctl;  // data warps + the control warp(s)
@@ -765,7 +779,7 @@ ccube_result_t allreduce_impl(void *const *bufs, size_t count, ccube_dtype_t dty
   a.sgd = g.sgd ? 1 : 0;
   a.sgd_alpha = g.sgd_alpha;
   a.tma = tma;
-  a.split_control = g.split_control;
+  a.split_control = nctl == 2 ? 1 : 0;
   a.backoff_ns = g.backoff_ns;
   a.debug_nodep = g.debug_nodep;
   a.elem_size = static_cast<int>(es);
@@ -1091,7 +1105,10 @@ ccube_result_t ccube_init(const ccube_world_t *world, ccube_tree_kind_t tree_kin
   g.transport = transport;
   g.overlap = 1;
   g.l2_hints = env_int("CCUBE_L2_HINTS", 1);
-  g.split_control = env_int("CCUBE_SPLIT_CONTROL", 1) != 0 ? 1 : 0;
+  {
+    const int sc = env_int("CCUBE_SPLIT_CONTROL", -1);
+    g.split_control = sc < 0 ? -1 : (sc != 0 ? 1 : 0);
+  }
   g.task_order = env_int("CCUBE_TASK_ORDER", 0);
   g.backoff_ns = env_int("CCUBE_BACKOFF_NS", 64);
   g.debug_nodep = env_int("CCUBE_DEBUG_NODEP", 0);
