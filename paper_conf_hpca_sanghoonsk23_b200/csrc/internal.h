@@ -28,6 +28,7 @@ namespace ccube {
 
 constexpr int kMaxRanks = 8;
 constexpr int kDefaultDataThreads = 192;  // data warps per CTA x 32 (CCUBE_THREADS)
+constexpr uint64_t kOneControlMinChunks = 128;  // AUTO control: one control warp from here
 constexpr int kMaxChannels = 128;
 constexpr int kMaxTrees = 8;  // ROTATED: one tree per rank
 constexpr int kMaxChildren = 2;

@@ -729,18 +729,20 @@ ccube_result_t allreduce_impl(void *const *bufs, size_t count, ccube_dtype_t dty
     // 3 KB blocks tile it; 8 data warps with 2 KB blocks when the slices are short
     // (many channels: P = 2 / 4), where fewer warps would mean fewer bytes in flight
     // (round 2).  In the 256-thread case AUTO control (CCUBE_SPLIT_CONTROL
-    // unset) runs ONE control warp and 7 data warps instead of 2 + 6: the data warps'
-    // registers are the bytes in flight, and the extra warp outweighs the poll round
-    // trip a release may now wait behind (P = 8: single 0.3191 -> 0.3166 ms, double
-    // 0.3236 -> 0.3141 ms, round 2 session 2).  Deterministic in agreed
-    // quantities, like J.
+    // unset) runs ONE control warp and 7 data warps instead of 2 + 6 once the call has
+    // >= kOneControlMinChunks chunks: the data warps' registers are the bytes in
+    // flight, and on a bandwidth-bound call the extra warp outweighs the poll round
+    // trip a release may now wait behind (P = 8, 102 MB: single 0.3191 -> 0.3166 ms,
+    // double 0.3236 -> 0.3141 ms), while a latency-bound one (<= 64 chunks: the fill
+    // and drain dominate) loses 4-10% to that round trip (round 2 session
+    // 2).  Deterministic in agreed quantities, like J.
     CC_TRY(capacity(kDefaultDataThreads, &cap, &tma));  // a 256-thread CTA (nctl = 2)
     const int J0 = g.channels ? g.channels : plan_auto_channels(in, cap);
     const uint64_t first = bytes < g.chunk_bytes ? bytes : g.chunk_bytes;
     const uint64_t units = (first + 2047) / 2048;
     if (units >= 3ull * J0) {
       data_threads = kDefaultDataThreads;
-      if (g.split_control < 0 && !split_heads_now()) {
+      if (g.split_control < 0 && !split_heads_now() && K >= kOneControlMinChunks) {
         nctl = 1;
         data_threads += 32;  // the same 256-thread CTA
       }
