@@ -117,8 +117,8 @@ typedef struct {
  *   CCUBE_DATAPATH, CCUBE_TRANSPORT, CCUBE_L2_HINTS, CCUBE_SPLIT_CONTROL) are part of
  *   the configuration every rank must share; ccube_init checks them.
  *   (CCUBE_SPLIT_CONTROL: unset = AUTO, one control warp + 7 data warps in the
- *   256-thread CTA geometry, the poll + publish pair otherwise; 1 / 0 force the
- *   pair / the single warp.)
+ *   256-thread CTA geometry on calls of >= 128 chunks, the poll + publish pair
+ *   otherwise; 1 / 0 force the pair / the single warp.)
  *   With several processes every tree neighbour on another GPU must be a CUDA peer
  *   (cudaDeviceCanAccessPeer), checked collectively. 
  * Errors: INVALID_ARG (bad world/tree/chunk, ranks disagree on the config or the
